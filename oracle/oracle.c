@@ -111,28 +111,45 @@ long oracle_arch_nparams(int arch) {
     return t;
 }
 
-/* Forward pass for one 112x50 input (row-major [row][feature]).
- * Activations are kept as act[position][channel].  Returns 0 on success. */
-int oracle_cnn_forward(int arch, int mode, const float* weights, long n_weights,
-                       const double* X, double* y_out) {
+/* Effective weights: the fp32 file values as double, rounded to bf16 for the
+ * tensor-core layers in ORACLE_BF16 mode (operand rounding, R16).  Done once
+ * per simulation; the same values are used for every instruction. */
+static double* effective_weights(int arch, int mode, const float* weights, long n) {
     layer_t L[16];
     int nl = arch_layers(arch, L);
-    if (nl < 0 || n_weights != oracle_arch_nparams(arch)) return -1;
+    double* W = (double*)malloc(sizeof(double) * (size_t)n);
+    long off = 0;
+    for (int li = 0; li < nl; li++) {
+        long nw = layer_nparams(&L[li]) - L[li].cout;          /* weights, then bias */
+        for (long t = 0; t < nw; t++) {
+            double v = (double)weights[off + t];
+            W[off + t] = (mode == ORACLE_BF16 && li != nl - 1) ? bf16_round(v) : v;
+        }
+        for (long t = nw; t < nw + L[li].cout; t++) W[off + t] = (double)weights[off + t];
+        off += nw + L[li].cout;
+    }
+    return W;
+}
 
-    /* buffers: positions x channels, at most 112 x 128 */
+/* Forward pass for one 112x50 input (row-major [row][feature]) with effective
+ * weights We.  Activations are kept as act[position][channel]. */
+static int forward(int arch, int mode, const double* We, const double* X, double* y_out) {
+    layer_t L[16];
+    int nl = arch_layers(arch, L);
+    if (nl < 0) return -1;
     static double cur[ORACLE_ROWS * 256], nxt[ORACLE_ROWS * 256], skip[ORACLE_ROWS * 256];
     int len = ORACLE_ROWS, ch = ORACLE_FEAT;
     for (int i = 0; i < len * ch; i++) cur[i] = X[i];
     int flat = 0; /* after the first linear the activation is a vector */
-    int skip_len = 0, skip_ch = 0;
-    const float* w = weights;
+    int skip_ch = 0;
+    const double* w = We;
 
     for (int li = 0; li < nl; li++) {
         const layer_t* l = &L[li];
         int tensor_core = (li != nl - 1);   /* R16: every layer but the last */
-        const float* Wt = w;
-        const float* B = w + (l->type == L_CONV ? (long)l->cout * l->cin * l->k
-                                                : (long)l->cout * l->cin);
+        const double* Wt = w;
+        const double* B = w + (l->type == L_CONV ? (long)l->cout * l->cin * l->k
+                                                 : (long)l->cout * l->cin);
         w += layer_nparams(l);
 
         /* operand rounding of the layer input (bf16 mode) */
@@ -141,7 +158,7 @@ int oracle_cnn_forward(int arch, int mode, const float* weights, long n_weights,
 
         if (l->res_begin) {                 /* remember block input x */
             for (int i = 0; i < len * ch; i++) skip[i] = cur[i];
-            skip_len = len; skip_ch = ch;
+            skip_ch = ch;
         }
 
         if (l->type == L_CONV) {
@@ -154,13 +171,10 @@ int oracle_cnn_forward(int arch, int mode, const float* weights, long n_weights,
                     for (int t = 0; t < l->k; t++) {
                         int r = p * l->stride + t - l->pad;
                         if (r < 0 || r >= len) continue;
-                        for (int c = 0; c < l->cin; c++) {
-                            double wv = Wt[((long)o * l->cin + c) * l->k + t];
-                            if (mode == ORACLE_BF16 && tensor_core) wv = bf16_round(wv);
-                            acc += wv * cur[r * ch + c];
-                        }
+                        for (int c = 0; c < l->cin; c++)
+                            acc += Wt[((long)o * l->cin + c) * l->k + t] * cur[r * ch + c];
                     }
-                    acc += (double)B[o];
+                    acc += B[o];
                     if (l->res_add) acc += skip[p * skip_ch + o];
                     if (l->relu && acc < 0.0) acc = 0.0;
                     nxt[p * l->cout + o] = acc;
@@ -172,23 +186,27 @@ int oracle_cnn_forward(int arch, int mode, const float* weights, long n_weights,
             if (nin != l->cin) return -2;
             for (int o = 0; o < l->cout; o++) {
                 double acc = 0.0;
-                for (int i = 0; i < nin; i++) {
-                    double wv = Wt[(long)o * l->cin + i];
-                    if (mode == ORACLE_BF16 && tensor_core) wv = bf16_round(wv);
-                    acc += wv * cur[i];
-                }
-                acc += (double)B[o];
+                for (int i = 0; i < nin; i++) acc += Wt[(long)o * l->cin + i] * cur[i];
+                acc += B[o];
                 if (l->relu && acc < 0.0) acc = 0.0;
                 nxt[o] = acc;
             }
             flat = 1; len = 1; ch = l->cout;
         }
-        (void)skip_len;
         memcpy(cur, nxt, sizeof(double) * (size_t)len * ch);
     }
     if (ch != 3) return -3;
     for (int i = 0; i < 3; i++) y_out[i] = cur[i];
     return 0;
+}
+
+int oracle_cnn_forward(int arch, int mode, const float* weights, long n_weights,
+                       const double* X, double* y_out) {
+    if (oracle_arch_nparams(arch) < 0 || n_weights != oracle_arch_nparams(arch)) return -1;
+    double* We = effective_weights(arch, mode, weights, n_weights);
+    int rc = forward(arch, mode, We, X, y_out);
+    free(We);
+    return rc;
 }
 
 /* Rounding of a predicted latency (R7): the double output is taken to
@@ -341,6 +359,7 @@ int oracle_simulate(int arch, int mode, const float* weights, long n_weights,
     if (cap < 1 || cap > ORACLE_MAXCAP) return -1;
     if (!forced_lat && n_weights != oracle_arch_nparams(arch)) return -2;
     double* X = (double*)malloc(sizeof(double) * ORACLE_ROWS * ORACLE_FEAT);
+    double* We = forced_lat ? NULL : effective_weights(arch, mode, weights, n_weights);
     int64_t total_stalls = 0;
     for (long j = j0; j < j0 + nj; j++) {
         int64_t s = (int64_t)(((__int128)j * L) / N);
@@ -355,8 +374,8 @@ int oracle_simulate(int arch, int mode, const float* weights, long n_weights,
             if (forced_lat) {
                 f = forced_lat[3 * i]; c = forced_lat[3 * i + 1]; st = forced_lat[3 * i + 2];
             } else {
-                if (oracle_cnn_forward(arch, mode, weights, n_weights, X, y) != 0) {
-                    free(X); oracle_queue_free(q); return -3;
+                if (forward(arch, mode, We, X, y) != 0) {
+                    free(X); free(We); oracle_queue_free(q); return -3;
                 }
                 f = oracle_round_latency(y[0]);
                 c = oracle_round_latency(y[1]);
@@ -378,5 +397,6 @@ int oracle_simulate(int arch, int mode, const float* weights, long n_weights,
     }
     if (stalls_out) *stalls_out = total_stalls;
     free(X);
+    free(We);
     return 0;
 }

@@ -1,0 +1,128 @@
+// internal.h -- product-side declarations shared by the libpsim translation
+// units.  Nothing here is visible through the C ABI (include/psim.h) and
+// nothing here is shared with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "psim.h"
+
+namespace psim {
+
+constexpr int kRows = 112;      // 111 instruction rows + 1 zero row (R11)
+constexpr int kFeat = 50;       // 3 time features + 47 attributes (R1)
+constexpr int kFeatPad = 64;    // device row width: features padded with zeros to 64
+constexpr int kQStride = 112;   // queue entries reserved per sub-trace (cap <= 110, +1 push)
+constexpr int kLatMax = 4095;   // R7
+constexpr int kTimeMax = 65535; // R7
+
+// One GEMM layer of the lowered CNN: out[M][N] = act(A[M][K] . W[N][K]^T + b[N]).
+// Convolutions with k = s = 2 read A as the row-pair reshape of the previous
+// activation [B*pos][C] -> [B*pos/2][2C] (K index = tap*C + channel), so no
+// im2col is ever materialised.
+struct GemmLayer {
+  int K = 0, N = 0;        // reduction length, output channels
+  int rows_per_item = 0;   // output positions per sub-trace (M = B * rows_per_item)
+  bool relu = true;
+  void* w = nullptr;       // device [N][K], fp32 or bf16 (K-major)
+  float* bias = nullptr;   // device [N] fp32
+  void* w_tc = nullptr;    // device weights pre-tiled for the tcgen05 kernel (bf16)
+};
+
+struct Model {
+  uint32_t arch = 0;
+  uint32_t precision = PSIM_FP32;
+  std::vector<GemmLayer> layers;  // tensor-core-able layers (all but the head)
+  float* head_w = nullptr;        // fc2 [3][256] fp32
+  float* head_b = nullptr;        // fc2 bias [3]
+  int head_in = 0;                // 256
+  bool loaded = false;
+};
+
+// Per-rank lockstep state: structure-of-arrays in HBM, sub-trace-major.
+struct SimState {
+  uint64_t n = 0;               // local sub-traces
+  int64_t* ws = nullptr;        // [n] first row (warm-up start)
+  int64_t* s = nullptr;         // [n] first real row
+  int64_t* e = nullptr;         // [n] end row
+  int64_t* clock = nullptr;     // [n] Clock
+  int64_t* bnd = nullptr;       // [n] Clock at the end of warm-up
+  int64_t* cycles = nullptr;    // [n] Clock_end - bnd
+  int32_t* count = nullptr;     // [n] live context entries
+  uint32_t* q_seq = nullptr;    // [n][kQStride] global row index of each live entry (fetch order)
+  uint32_t* q_fetch = nullptr;  // [n][kQStride] low 32 bits of the fetch Clock
+  uint32_t* q_cs = nullptr;     // [n][kQStride] c | s << 16
+  unsigned long long* k_hist = nullptr;   // [112]
+  unsigned long long* stalls = nullptr;   // [1]
+  long long* total = nullptr;             // [1] local sum of cycles (NCCL send/recv buffer)
+};
+
+struct Buffers {
+  size_t bytes = 0;
+  void* x = nullptr;            // gathered inputs [n][112][64] (fp32 or bf16)
+  void* act[6] = {};            // per-layer activations
+  float* h = nullptr;           // fc1 output [n][256] fp32
+  float* y = nullptr;           // head output [n][3] fp32
+};
+
+// ----------------------------- kernels ---------------------------------
+struct GatherArgs {
+  const uint8_t* trace;      // device rows, row r at trace + (r - row_lo) * stride
+  int64_t row_lo;
+  int64_t stride;
+  const int64_t* ws;
+  const int64_t* e;
+  const int64_t* clock;
+  const int32_t* count;
+  const uint32_t* q_seq;
+  const uint32_t* q_fetch;
+  const uint32_t* q_cs;
+  uint64_t n;
+  int64_t step;
+};
+void launch_gather_f32(const GatherArgs& a, float* x, cudaStream_t st);
+void launch_gather_bf16(const GatherArgs& a, __nv_bfloat16* x, cudaStream_t st);
+
+struct UpdateArgs {
+  SimState st;
+  int64_t row_lo;
+  int64_t step;
+  int cap;
+  const float* y;            // [n][3] raw CNN outputs (CNN mode) or nullptr
+  const uint16_t* forced;    // [rows][3] teacher-forced latencies (row - row_lo) or nullptr
+  uint16_t* rec_lat;         // [rows][3] or nullptr (PSIM_RECORD_ROWS)
+  int32_t* rec_k;            // [rows] or nullptr
+  int64_t* rec_clock;        // [rows] or nullptr
+};
+void launch_update(const UpdateArgs& a, cudaStream_t st);
+void launch_state_init(const SimState& s, cudaStream_t st);
+void launch_reduce_cycles(const SimState& s, cudaStream_t st);
+
+// head: y[b][o] = sum_i h[b][i] * w[o][i] + bias[o] (fp32, o < 3)
+void launch_head(const float* h, const float* w, const float* b, int in, float* y, uint64_t n,
+                 cudaStream_t st);
+
+// SIMT GEMM (CUDA cores): C = act(A . W^T + b); A [M][K], W [N][K]
+void launch_gemm_simt_f32(const float* A, const float* W, const float* b, float* C, int64_t M,
+                          int N, int K, bool relu, cudaStream_t st);
+void launch_gemm_simt_bf16(const __nv_bfloat16* A, const __nv_bfloat16* W, const float* b,
+                           void* C, bool c_is_f32, int64_t M, int N, int K, bool relu,
+                           cudaStream_t st);
+
+// tcgen05 GEMM (tensor cores, sm_100a): bf16 A/W, fp32 accumulate in TMEM.
+// Returns false if the shape is not supported by the tensor-core kernel.
+bool gemm_tc_supported(int N, int K);
+void launch_gemm_tc(const __nv_bfloat16* A, const void* Wtc, const float* b, void* C,
+                    bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st);
+// Pre-tile a [N][K] bf16 weight for the tensor-core kernel (device -> device).
+void* pretile_weight_tc(const __nv_bfloat16* W, int N, int K, cudaStream_t st);
+
+// pad/convert the caller's [B][112][50] fp32 inputs (psim_cnn_forward)
+void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st);
+
+}  // namespace psim

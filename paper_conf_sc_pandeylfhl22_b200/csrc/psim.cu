@@ -1,0 +1,632 @@
+// psim.cu -- host runtime behind the C ABI (include/psim.h): context and
+// state machine, partitioner, trace loader, model repacking, the lockstep
+// step loop and the end-of-run NCCL reduction.
+//
+// Step t (PAPER.md:91-107 per instruction, lockstep over sub-traces :179):
+//   gather -> conv/fc GEMMs -> head (fc2) -> update (round, Clock, retire, push)
+// After the last step: reduce cycles, ncclAllReduce(int64, sum).
+#include <dlfcn.h>
+#include <nccl.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+using namespace psim;
+
+namespace {
+// ---- NCCL, resolved at run time (the library never links a specific NCCL) ----
+struct NcclApi {
+  bool tried = false, ok = false;
+  ncclResult_t (*commInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+  const char* (*errStr)(ncclResult_t) = nullptr;
+};
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+
+bool load_nccl() {
+  std::lock_guard<std::mutex> lk(g_nccl_mu);
+  if (g_nccl.tried) return g_nccl.ok;
+  g_nccl.tried = true;
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+  if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) return false;
+  g_nccl.commInitRank = (decltype(g_nccl.commInitRank))dlsym(h, "ncclCommInitRank");
+  g_nccl.allReduce = (decltype(g_nccl.allReduce))dlsym(h, "ncclAllReduce");
+  g_nccl.commDestroy = (decltype(g_nccl.commDestroy))dlsym(h, "ncclCommDestroy");
+  g_nccl.errStr = (decltype(g_nccl.errStr))dlsym(h, "ncclGetErrorString");
+  g_nccl.ok = g_nccl.commInitRank && g_nccl.allReduce && g_nccl.commDestroy && g_nccl.errStr;
+  return g_nccl.ok;
+}
+
+inline uint16_t f32_to_bf16_rne(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  if ((u & 0x7f800000u) == 0x7f800000u && (u & 0x7fffffu)) return (uint16_t)((u >> 16) | 0x40);  // NaN
+  u += 0x7fffu + ((u >> 16) & 1u);
+  return (uint16_t)(u >> 16);
+}
+}  // namespace
+
+struct psim_ctx {
+  psim_opts opts{};
+  int cap = 110;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  std::string err;
+  // trace
+  bool have_trace = false;
+  const uint8_t* trace = nullptr;
+  uint64_t L = 0, first_row = 0, n_rows = 0, stride = 48;
+  int trace_mode = 0;
+  uint8_t* d_trace = nullptr;
+  size_t d_trace_cap = 0;
+  // partition
+  bool partitioned = false;
+  uint64_t N = 0, W = 0, j0 = 0, j1 = 0;
+  int64_t row_lo = 0, row_hi = 0, steps = 0;
+  std::vector<int64_t> h_ws, h_s, h_e;
+  // model / forcing
+  Model model;
+  std::vector<uint16_t> forced;
+  uint16_t* d_forced = nullptr;
+  size_t d_forced_cap = 0;
+  // state
+  SimState st{};
+  uint64_t st_cap = 0;
+  Buffers buf{};
+  uint64_t buf_n = 0;
+  uint16_t* rec_lat = nullptr;
+  int32_t* rec_k = nullptr;
+  int64_t* rec_clock = nullptr;
+  size_t rec_cap = 0;
+  // results
+  bool done = false;
+  int64_t total = 0;
+  psim_stats stats{};
+  ncclComm_t comm = nullptr;
+  cudaEvent_t ev[4] = {};
+};
+
+#define FAIL(code, ...)                                   \
+  do {                                                    \
+    char _b[512];                                         \
+    snprintf(_b, sizeof _b, __VA_ARGS__);                 \
+    ctx->err = _b;                                        \
+    return code;                                          \
+  } while (0)
+#define CK(x)                                                                              \
+  do {                                                                                     \
+    cudaError_t _e = (x);                                                                  \
+    if (_e != cudaSuccess) FAIL(_e == cudaErrorMemoryAllocation ? PSIM_ERR_OOM : PSIM_ERR_CUDA, \
+                                "%s failed: %s (%s:%d)", #x, cudaGetErrorString(_e), __FILE__, __LINE__); \
+  } while (0)
+
+static void dfree(void* p) {
+  if (p) cudaFree(p);
+}
+
+extern "C" {
+
+const char* psim_version(void) {
+  return "psim 0.1 (sm_100a; gather/update warp-per-sub-trace, GEMM: tcgen05+TMA bf16, SIMT fp32)";
+}
+
+int psim_create(const psim_opts* opts, psim_ctx** out) {
+  if (!out) return PSIM_ERR_ARG;
+  *out = nullptr;
+  if (!opts) return PSIM_ERR_ARG;
+  if (opts->world_size < 1 || opts->rank < 0 || opts->rank >= opts->world_size) return PSIM_ERR_ARG;
+  if (opts->queue_cap > PSIM_MAX_CAP) return PSIM_ERR_ARG;
+  if (opts->precision != PSIM_FP32 && opts->precision != PSIM_BF16) return PSIM_ERR_ARG;
+  psim_ctx* ctx = new psim_ctx();
+  ctx->opts = *opts;
+  ctx->cap = opts->queue_cap ? (int)opts->queue_cap : (int)PSIM_MAX_CAP;
+  if (cudaSetDevice(opts->device) != cudaSuccess) { delete ctx; return PSIM_ERR_CUDA; }
+  if (opts->stream) {
+    ctx->stream = (cudaStream_t)opts->stream;
+  } else {
+    if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) { delete ctx; return PSIM_ERR_CUDA; }
+    ctx->own_stream = true;
+  }
+  for (auto& e : ctx->ev) cudaEventCreate(&e);
+  if (opts->world_size > 1 && opts->nccl_id) {
+    if (!load_nccl()) { psim_destroy(ctx); return PSIM_ERR_NCCL; }
+    ncclUniqueId id;
+    memcpy(&id, opts->nccl_id, sizeof id);
+    if (g_nccl.commInitRank(&ctx->comm, opts->world_size, id, opts->rank) != ncclSuccess) {
+      ctx->comm = nullptr;
+      psim_destroy(ctx);
+      return PSIM_ERR_NCCL;
+    }
+  }
+  *out = ctx;
+  return PSIM_OK;
+}
+
+void psim_destroy(psim_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->opts.device);
+  if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+  if (ctx->comm && g_nccl.ok) g_nccl.commDestroy(ctx->comm);
+  dfree(ctx->d_trace);
+  dfree(ctx->d_forced);
+  for (auto& l : ctx->model.layers) { dfree(l.w); dfree(l.bias); }
+  dfree(ctx->model.head_w);
+  dfree(ctx->model.head_b);
+  SimState& s = ctx->st;
+  for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
+                  (void*)s.count, (void*)s.q_seq, (void*)s.q_fetch, (void*)s.q_cs, (void*)s.k_hist,
+                  (void*)s.stalls, (void*)s.total})
+    dfree(p);
+  dfree(ctx->buf.x);
+  for (void* p : ctx->buf.act) dfree(p);
+  dfree(ctx->buf.h);
+  dfree(ctx->buf.y);
+  dfree(ctx->rec_lat);
+  dfree(ctx->rec_k);
+  dfree(ctx->rec_clock);
+  for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
+  if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
+  delete ctx;
+}
+
+const char* psim_last_error(const psim_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+int psim_load_trace(psim_ctx* ctx, const uint8_t* attrs, uint64_t n_instr, uint64_t first_row,
+                    uint64_t n_rows, uint32_t n_attr, uint64_t row_stride) {
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!attrs || n_instr == 0) FAIL(PSIM_ERR_ARG, "empty trace");
+  if (n_instr >= (1ull << 32)) FAIL(PSIM_ERR_ARG, "L must be < 2^32 (row indices are uint32)");
+  if (n_attr != PSIM_NATTR) FAIL(PSIM_ERR_ARG, "n_attr must be 47, got %u", n_attr);
+  if (row_stride < 48) FAIL(PSIM_ERR_ARG, "row_stride must be >= 48");
+  if (n_rows == 0 || first_row + n_rows > n_instr) FAIL(PSIM_ERR_ARG, "rows [%llu,%llu) outside [0,%llu)",
+                                                         (unsigned long long)first_row,
+                                                         (unsigned long long)(first_row + n_rows),
+                                                         (unsigned long long)n_instr);
+  cudaPointerAttributes pa{};
+  int mode = 2;
+  if (cudaPointerGetAttributes(&pa, attrs) == cudaSuccess) {
+    if (pa.type == cudaMemoryTypeDevice || pa.type == cudaMemoryTypeManaged) mode = 0;
+    else if (pa.type == cudaMemoryTypeHost) mode = 1;
+  }
+  cudaGetLastError();
+  if (mode == 0 && (row_stride % 16)) FAIL(PSIM_ERR_ARG, "device trace row_stride must be a multiple of 16");
+  if (ctx->L != n_instr) ctx->partitioned = false;
+  ctx->trace = attrs;
+  ctx->L = n_instr;
+  ctx->first_row = first_row;
+  ctx->n_rows = n_rows;
+  ctx->stride = row_stride;
+  ctx->trace_mode = mode;
+  ctx->have_trace = true;
+  ctx->done = false;
+  return PSIM_OK;
+}
+
+// Rank g of G owns sub-traces [floor(gN/G), floor((g+1)N/G)); sub-trace j is
+// [s_j, e_j) with s_j = floor(jL/N) (R8) and warm-up start max(0, s_j - W) (R9).
+static void rank_block(uint64_t L, uint64_t N, uint64_t W, int g, int G, std::vector<int64_t>* ws_,
+                       std::vector<int64_t>* s_, std::vector<int64_t>* e_, uint64_t* j0p, uint64_t* j1p,
+                       int64_t* lop, int64_t* hip, int64_t* stepsp) {
+  const uint64_t j0 = (uint64_t)(((unsigned __int128)g * N) / G);
+  const uint64_t j1 = (uint64_t)(((unsigned __int128)(g + 1) * N) / G);
+  auto sj = [&](uint64_t j) { return (int64_t)(((unsigned __int128)j * L) / N); };
+  int64_t lo = INT64_MAX, hi = 0, steps = 0;
+  for (uint64_t j = j0; j < j1; ++j) {
+    const int64_t s = sj(j), e = sj(j + 1);
+    const int64_t ws = s > (int64_t)W ? s - (int64_t)W : 0;
+    if (ws_) { ws_->push_back(ws); s_->push_back(s); e_->push_back(e); }
+    lo = std::min(lo, ws); hi = std::max(hi, e);
+    steps = std::max(steps, e - ws);
+  }
+  if (j1 == j0) { lo = 0; hi = 0; }
+  *j0p = j0; *j1p = j1; *lop = lo; *hip = hi; *stepsp = steps;
+}
+
+int psim_partition_range(uint64_t L, uint64_t N, uint64_t W, int rank, int world, uint64_t* j0,
+                         uint64_t* j1, uint64_t* row_lo, uint64_t* row_hi, uint64_t* steps) {
+  if (N == 0 || N > L || world < 1 || rank < 0 || rank >= world) return PSIM_ERR_ARG;
+  uint64_t a, b;
+  int64_t lo, hi, st;
+  rank_block(L, N, W, rank, world, nullptr, nullptr, nullptr, &a, &b, &lo, &hi, &st);
+  if (j0) *j0 = a;
+  if (j1) *j1 = b;
+  if (row_lo) *row_lo = (uint64_t)lo;
+  if (row_hi) *row_hi = (uint64_t)hi;
+  if (steps) *steps = (uint64_t)st;
+  return PSIM_OK;
+}
+
+int psim_partition(psim_ctx* ctx, uint64_t N, uint64_t W) {
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->have_trace) FAIL(PSIM_ERR_STATE, "partition before load_trace");
+  const uint64_t L = ctx->L;
+  if (N == 0 || N > L) FAIL(PSIM_ERR_ARG, "need 1 <= N <= L (N=%llu, L=%llu)", (unsigned long long)N,
+                            (unsigned long long)L);
+  const int G = ctx->opts.world_size, g = ctx->opts.rank;
+  ctx->h_ws.clear(); ctx->h_s.clear(); ctx->h_e.clear();
+  uint64_t j0, j1;
+  int64_t lo, hi, steps;
+  rank_block(L, N, W, g, G, &ctx->h_ws, &ctx->h_s, &ctx->h_e, &j0, &j1, &lo, &hi, &steps);
+  if (j1 > j0 && ((uint64_t)lo < ctx->first_row || (uint64_t)hi > ctx->first_row + ctx->n_rows))
+    FAIL(PSIM_ERR_ARG, "loaded rows [%llu,%llu) do not cover this rank's range [%lld,%lld)",
+         (unsigned long long)ctx->first_row, (unsigned long long)(ctx->first_row + ctx->n_rows),
+         (long long)lo, (long long)hi);
+  ctx->N = N; ctx->W = W; ctx->j0 = j0; ctx->j1 = j1;
+  ctx->row_lo = lo; ctx->row_hi = hi; ctx->steps = steps;
+  ctx->partitioned = true;
+  ctx->done = false;
+  return PSIM_OK;
+}
+
+int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, uint64_t n_floats) {
+  if (!ctx || !desc || !w) return PSIM_ERR_ARG;
+  if (desc->rows != 112 || desc->features != 50) FAIL(PSIM_ERR_ARG, "model input must be 112 x 50");
+  struct L_ { int kind, cin, cout, k; };   // kind 0 conv, 1 linear
+  std::vector<L_> ls;
+  if (desc->arch == PSIM_ARCH_M2) ls = {{0, 50, 64, 2}, {0, 64, 64, 2}, {1, 1792, 256, 0}, {1, 256, 3, 0}};
+  else if (desc->arch == PSIM_ARCH_C3) ls = {{0, 50, 64, 2}, {0, 64, 128, 2}, {0, 128, 128, 2}, {1, 1792, 256, 0}, {1, 256, 3, 0}};
+  else if (desc->arch == PSIM_ARCH_RB7) FAIL(PSIM_ERR_UNSUPPORTED, "RB7 is not built in this round");
+  else FAIL(PSIM_ERR_ARG, "unknown arch %u", desc->arch);
+  uint64_t need = 0;
+  for (auto& l : ls) need += (uint64_t)l.cout * l.cin * (l.kind == 0 ? l.k : 1) + l.cout;
+  if (need != n_floats) FAIL(PSIM_ERR_ARG, "weight count %llu != %llu for arch %u", (unsigned long long)n_floats,
+                             (unsigned long long)need, desc->arch);
+  CK(cudaSetDevice(ctx->opts.device));
+  Model& m = ctx->model;
+  for (auto& l : m.layers) { dfree(l.w); dfree(l.bias); }
+  m.layers.clear();
+  dfree(m.head_w); dfree(m.head_b);
+  m.head_w = m.head_b = nullptr;
+  const bool bf16 = ctx->opts.precision == PSIM_BF16;
+  const float* p = w;
+  int pos = 112;   // current positions
+  int ch = 50;     // current channels (device layout pads 50 -> 64)
+  for (size_t li = 0; li < ls.size(); ++li) {
+    const L_& l = ls[li];
+    const float* W = p;
+    const float* B = p + (uint64_t)l.cout * l.cin * (l.kind == 0 ? l.k : 1);
+    p = B + l.cout;
+    if (li == ls.size() - 1) {   // head: fc2 stays fp32 (R16)
+      CK(cudaMalloc(&m.head_w, sizeof(float) * 3 * l.cin));
+      CK(cudaMalloc(&m.head_b, sizeof(float) * 3));
+      CK(cudaMemcpy(m.head_w, W, sizeof(float) * 3 * l.cin, cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(m.head_b, B, sizeof(float) * 3, cudaMemcpyHostToDevice));
+      m.head_in = l.cin;
+      break;
+    }
+    GemmLayer g;
+    std::vector<float> Wk;
+    if (l.kind == 0) {
+      // conv k=s=2: K index = tap * Cin_dev + channel (Cin_dev = 64 for the first layer)
+      const int cin_dev = (li == 0) ? kFeatPad : l.cin;
+      g.K = 2 * cin_dev;
+      g.N = l.cout;
+      Wk.assign((size_t)g.N * g.K, 0.f);
+      for (int o = 0; o < l.cout; ++o)
+        for (int c = 0; c < l.cin; ++c)
+          for (int t = 0; t < 2; ++t) Wk[(size_t)o * g.K + t * cin_dev + c] = W[((size_t)o * l.cin + c) * 2 + t];
+      pos /= 2;
+      g.rows_per_item = pos;
+      ch = l.cout;
+    } else {
+      if (l.cin != pos * ch) FAIL(PSIM_ERR_ARG, "internal: fc1 fan-in %d != %d", l.cin, pos * ch);
+      g.K = l.cin;
+      g.N = l.cout;
+      Wk.assign(W, W + (size_t)g.N * g.K);   // position-major already (R11)
+      g.rows_per_item = 1;
+      pos = 1;
+      ch = l.cout;
+    }
+    g.relu = true;
+    CK(cudaMalloc(&g.bias, sizeof(float) * g.N));
+    CK(cudaMemcpy(g.bias, B, sizeof(float) * g.N, cudaMemcpyHostToDevice));
+    if (bf16) {
+      std::vector<uint16_t> wb(Wk.size());
+      for (size_t t = 0; t < Wk.size(); ++t) wb[t] = f32_to_bf16_rne(Wk[t]);
+      CK(cudaMalloc(&g.w, wb.size() * 2));
+      CK(cudaMemcpy(g.w, wb.data(), wb.size() * 2, cudaMemcpyHostToDevice));
+      if (gemm_tc_supported(g.N, g.K)) {
+        g.w_tc = pretile_weight_tc((const __nv_bfloat16*)g.w, g.N, g.K, ctx->stream);
+        CK(cudaStreamSynchronize(ctx->stream));
+        CK(cudaGetLastError());
+      }
+    } else {
+      CK(cudaMalloc(&g.w, Wk.size() * 4));
+      CK(cudaMemcpy(g.w, Wk.data(), Wk.size() * 4, cudaMemcpyHostToDevice));
+    }
+    m.layers.push_back(g);
+  }
+  m.arch = desc->arch;
+  m.precision = ctx->opts.precision;
+  m.loaded = true;
+  ctx->done = false;
+  return PSIM_OK;
+}
+
+int psim_force_latencies(psim_ctx* ctx, const uint16_t* lat3, uint64_t n_instr) {
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!lat3) { ctx->forced.clear(); return PSIM_OK; }
+  if (!ctx->have_trace || n_instr != ctx->L) FAIL(PSIM_ERR_ARG, "forced latencies must cover all L rows");
+  ctx->forced.assign(lat3, lat3 + 3 * n_instr);
+  ctx->done = false;
+  return PSIM_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------
+static int ensure_buffers(psim_ctx* ctx, uint64_t n) {
+  const bool bf16 = ctx->opts.precision == PSIM_BF16;
+  const size_t es = bf16 ? 2 : 4;
+  if (ctx->buf_n >= n && ctx->buf.x) return PSIM_OK;
+  dfree(ctx->buf.x);
+  for (void*& p : ctx->buf.act) { dfree(p); p = nullptr; }
+  dfree(ctx->buf.h);
+  dfree(ctx->buf.y);
+  ctx->buf = Buffers{};
+  CK(cudaMalloc(&ctx->buf.x, n * kRows * kFeatPad * es));
+  CK(cudaMemset(ctx->buf.x, 0, n * kRows * kFeatPad * es));
+  for (size_t li = 0; li + 1 < ctx->model.layers.size(); ++li) {
+    const GemmLayer& g = ctx->model.layers[li];
+    CK(cudaMalloc(&ctx->buf.act[li], n * g.rows_per_item * g.N * es));
+  }
+  CK(cudaMalloc(&ctx->buf.h, n * 256 * sizeof(float)));
+  CK(cudaMalloc(&ctx->buf.y, n * 3 * sizeof(float)));
+  ctx->buf_n = n;
+  return PSIM_OK;
+}
+
+// Run the lowered CNN on buf.x (n items) -> buf.y.  Counts launches.
+static int run_cnn(psim_ctx* ctx, uint64_t n, uint64_t* launches) {
+  const Model& m = ctx->model;
+  const bool bf16 = m.precision == PSIM_BF16;
+  const void* in = ctx->buf.x;
+  for (size_t li = 0; li < m.layers.size(); ++li) {
+    const GemmLayer& g = m.layers[li];
+    const bool last = li + 1 == m.layers.size();
+    void* out = last ? (void*)ctx->buf.h : ctx->buf.act[li];
+    const int64_t M = (int64_t)n * g.rows_per_item;
+    if (bf16) {
+      if (g.w_tc) launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
+      else launch_gemm_simt_bf16((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
+    } else {
+      launch_gemm_simt_f32((const float*)in, (const float*)g.w, g.bias, (float*)out, M, g.N, g.K, g.relu, ctx->stream);
+    }
+    (*launches)++;
+    in = out;
+  }
+  launch_head(ctx->buf.h, m.head_w, m.head_b, m.head_in, ctx->buf.y, n, ctx->stream);
+  (*launches)++;
+  return PSIM_OK;
+}
+
+extern "C" int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float* Y) {
+  if (!ctx || !X || !Y || B == 0) return PSIM_ERR_ARG;
+  if (!ctx->model.loaded) FAIL(PSIM_ERR_STATE, "load_model first");
+  CK(cudaSetDevice(ctx->opts.device));
+  int rc = ensure_buffers(ctx, B);
+  if (rc) return rc;
+  float* dX = nullptr;
+  CK(cudaMalloc(&dX, B * kRows * kFeat * sizeof(float)));
+  cudaError_t e = cudaMemcpyAsync(dX, X, B * kRows * kFeat * sizeof(float), cudaMemcpyHostToDevice, ctx->stream);
+  if (e == cudaSuccess) {
+    launch_pad_inputs(dX, B, ctx->buf.x, ctx->model.precision == PSIM_BF16, ctx->stream);
+    uint64_t l = 0;
+    run_cnn(ctx, B, &l);
+    e = cudaMemcpyAsync(Y, ctx->buf.y, B * 3 * sizeof(float), cudaMemcpyDeviceToHost, ctx->stream);
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+  if (e == cudaSuccess) e = cudaGetLastError();
+  cudaFree(dX);
+  CK(e);
+  return PSIM_OK;
+}
+
+static int ensure_state(psim_ctx* ctx) {
+  const uint64_t n = ctx->j1 - ctx->j0;
+  SimState& s = ctx->st;
+  if (ctx->st_cap < n || !s.clock) {
+    for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
+                    (void*)s.count, (void*)s.q_seq, (void*)s.q_fetch, (void*)s.q_cs})
+      dfree(p);
+    const uint64_t a = std::max<uint64_t>(n, 1);
+    CK(cudaMalloc(&s.ws, a * 8)); CK(cudaMalloc(&s.s, a * 8)); CK(cudaMalloc(&s.e, a * 8));
+    CK(cudaMalloc(&s.clock, a * 8)); CK(cudaMalloc(&s.bnd, a * 8)); CK(cudaMalloc(&s.cycles, a * 8));
+    CK(cudaMalloc(&s.count, a * 4));
+    CK(cudaMalloc(&s.q_seq, a * kQStride * 4)); CK(cudaMalloc(&s.q_fetch, a * kQStride * 4));
+    CK(cudaMalloc(&s.q_cs, a * kQStride * 4));
+    ctx->st_cap = a;
+  }
+  if (!s.k_hist) {
+    CK(cudaMalloc(&s.k_hist, 112 * 8));
+    CK(cudaMalloc(&s.stalls, 8));
+    CK(cudaMalloc(&s.total, 8));
+  }
+  s.n = n;
+  if (n) {
+    CK(cudaMemcpyAsync(s.ws, ctx->h_ws.data(), n * 8, cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaMemcpyAsync(s.s, ctx->h_s.data(), n * 8, cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaMemcpyAsync(s.e, ctx->h_e.data(), n * 8, cudaMemcpyHostToDevice, ctx->stream));
+  }
+  return PSIM_OK;
+}
+
+extern "C" int psim_simulate(psim_ctx* ctx) {
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->have_trace || !ctx->partitioned) FAIL(PSIM_ERR_STATE, "simulate needs load_trace and partition");
+  const bool forced = !ctx->forced.empty();
+  if (!forced && !ctx->model.loaded) FAIL(PSIM_ERR_STATE, "simulate needs load_model or force_latencies");
+  CK(cudaSetDevice(ctx->opts.device));
+  cudaStream_t st = ctx->stream;
+  const uint64_t n = ctx->j1 - ctx->j0;
+  const int64_t rows = ctx->row_hi - ctx->row_lo;
+  uint64_t launches = 0;
+  psim_stats stats{};
+  stats.subtraces = n;
+  stats.trace_mode = ctx->trace_mode;
+
+  int rc = ensure_state(ctx);
+  if (rc) return rc;
+  if (!forced) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
+  const bool rec = (ctx->opts.flags & PSIM_RECORD_ROWS) != 0;
+  if (rec && ctx->rec_cap < (size_t)rows) {
+    dfree(ctx->rec_lat); dfree(ctx->rec_k); dfree(ctx->rec_clock);
+    CK(cudaMalloc(&ctx->rec_lat, rows * 6 + 8));
+    CK(cudaMalloc(&ctx->rec_k, rows * 4 + 8));
+    CK(cudaMalloc(&ctx->rec_clock, rows * 8 + 8));
+    ctx->rec_cap = rows;
+  }
+  if (forced) {
+    if (ctx->d_forced_cap < (size_t)rows) {
+      dfree(ctx->d_forced);
+      CK(cudaMalloc(&ctx->d_forced, rows * 6 + 8));
+      ctx->d_forced_cap = rows;
+    }
+    CK(cudaMemcpyAsync(ctx->d_forced, ctx->forced.data() + 3 * ctx->row_lo, rows * 6, cudaMemcpyHostToDevice, st));
+  }
+
+  // ---- trace: the rank's rows cross the host link once ----
+  CK(cudaEventRecord(ctx->ev[0], st));
+  const uint8_t* dtr;
+  if (ctx->trace_mode == 0) {
+    dtr = ctx->trace + (ctx->row_lo - (int64_t)ctx->first_row) * ctx->stride;
+  } else {
+    const size_t bytes = (size_t)rows * ctx->stride;
+    if (ctx->d_trace_cap < bytes) {
+      dfree(ctx->d_trace);
+      ctx->d_trace = nullptr;
+      CK(cudaMalloc(&ctx->d_trace, bytes + 64));
+      ctx->d_trace_cap = bytes;
+    }
+    if (bytes)
+      CK(cudaMemcpyAsync(ctx->d_trace, ctx->trace + (ctx->row_lo - (int64_t)ctx->first_row) * ctx->stride, bytes,
+                         cudaMemcpyHostToDevice, st));
+    stats.h2d_bytes = bytes;
+    dtr = ctx->d_trace;
+  }
+  CK(cudaEventRecord(ctx->ev[1], st));
+
+  launch_state_init(ctx->st, st);
+  launches++;
+  const bool bf16 = ctx->model.precision == PSIM_BF16;
+  GatherArgs ga{dtr, ctx->row_lo, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e, ctx->st.clock, ctx->st.count,
+                ctx->st.q_seq, ctx->st.q_fetch, ctx->st.q_cs, n, 0};
+  UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, forced ? nullptr : ctx->buf.y,
+                forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
+                rec ? ctx->rec_clock : nullptr};
+  for (int64_t t = 0; t < ctx->steps && n; ++t) {
+    if (!forced) {
+      ga.step = t;
+      if (bf16) launch_gather_bf16(ga, (__nv_bfloat16*)ctx->buf.x, st);
+      else launch_gather_f32(ga, (float*)ctx->buf.x, st);
+      launches++;
+      rc = run_cnn(ctx, n, &launches);
+      if (rc) return rc;
+    }
+    ua.step = t;
+    launch_update(ua, st);
+    launches++;
+  }
+  launch_reduce_cycles(ctx->st, st);
+  launches++;
+  CK(cudaGetLastError());
+  if (ctx->comm) {
+    ncclResult_t r = g_nccl.allReduce(ctx->st.total, ctx->st.total, 1, ncclInt64, ncclSum, ctx->comm, st);
+    if (r != ncclSuccess) FAIL(PSIM_ERR_NCCL, "ncclAllReduce: %s", g_nccl.errStr(r));
+  }
+  CK(cudaEventRecord(ctx->ev[2], st));
+  long long total = 0;
+  CK(cudaMemcpyAsync(&total, ctx->st.total, 8, cudaMemcpyDeviceToHost, st));
+  unsigned long long hist[112], stalls = 0;
+  CK(cudaMemcpyAsync(hist, ctx->st.k_hist, sizeof hist, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&stalls, ctx->st.stalls, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  CK(cudaGetLastError());
+  float ms_all = 0, ms_load = 0;
+  cudaEventElapsedTime(&ms_all, ctx->ev[0], ctx->ev[2]);
+  cudaEventElapsedTime(&ms_load, ctx->ev[0], ctx->ev[1]);
+  ctx->total = total;
+  for (int k = 0; k < 112; ++k) stats.k_hist[k] = hist[k];
+  stats.stalls = stalls;
+  stats.steps = (uint64_t)ctx->steps;
+  uint64_t sim = 0, cnt = 0;
+  for (uint64_t b = 0; b < n; ++b) { sim += ctx->h_e[b] - ctx->h_ws[b]; cnt += ctx->h_e[b] - ctx->h_s[b]; }
+  stats.simulated = sim;
+  stats.counted = cnt;
+  stats.gpu_launches = launches;
+  stats.sim_ms = ms_all;
+  stats.load_ms = ms_load;
+  if (ctx->comm == nullptr) stats.local_cycles = total;
+  else {
+    long long lc = 0;
+    // local sum = re-reduce the cycles (cheap; diagnostics only)
+    std::vector<long long> cyc(n);
+    if (n) CK(cudaMemcpy(cyc.data(), ctx->st.cycles, n * 8, cudaMemcpyDeviceToHost));
+    for (auto v : cyc) lc += v;
+    stats.local_cycles = lc;
+  }
+  ctx->stats = stats;
+  ctx->done = true;
+  return PSIM_OK;
+}
+
+extern "C" int psim_total_cycles(const psim_ctx* ctx, int64_t* out) {
+  if (!ctx || !out) return PSIM_ERR_ARG;
+  if (!ctx->done) return PSIM_ERR_STATE;
+  *out = ctx->total;
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_rows(const psim_ctx* cctx, uint64_t first, uint64_t n, uint16_t* out3, int32_t* k,
+                             int64_t* clock) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (!(ctx->opts.flags & PSIM_RECORD_ROWS)) FAIL(PSIM_ERR_STATE, "context created without PSIM_RECORD_ROWS");
+  const int64_t s_first = ctx->h_s.empty() ? 0 : ctx->h_s.front();
+  if ((int64_t)first < s_first || (int64_t)(first + n) > ctx->row_hi) FAIL(PSIM_ERR_ARG, "rows outside this rank");
+  const int64_t off = (int64_t)first - ctx->row_lo;
+  CK(cudaSetDevice(ctx->opts.device));
+  if (out3) CK(cudaMemcpy(out3, ctx->rec_lat + 3 * off, n * 6, cudaMemcpyDeviceToHost));
+  if (k) CK(cudaMemcpy(k, ctx->rec_k + off, n * 4, cudaMemcpyDeviceToHost));
+  if (clock) CK(cudaMemcpy(clock, ctx->rec_clock + off, n * 8, cudaMemcpyDeviceToHost));
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_subtrace_cycles(const psim_ctx* cctx, uint64_t first, uint64_t n, int64_t* out) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx || !out) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (first + n > ctx->j1 - ctx->j0) FAIL(PSIM_ERR_ARG, "sub-traces outside this rank");
+  CK(cudaSetDevice(ctx->opts.device));
+  CK(cudaMemcpy(out, ctx->st.cycles + first, n * 8, cudaMemcpyDeviceToHost));
+  return PSIM_OK;
+}
+
+extern "C" int psim_rank_range(const psim_ctx* ctx, uint64_t* j0, uint64_t* j1, uint64_t* lo, uint64_t* hi) {
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->partitioned) return PSIM_ERR_STATE;
+  if (j0) *j0 = ctx->j0;
+  if (j1) *j1 = ctx->j1;
+  if (lo) *lo = (uint64_t)ctx->row_lo;
+  if (hi) *hi = (uint64_t)ctx->row_hi;
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_stats(const psim_ctx* ctx, psim_stats* out) {
+  if (!ctx || !out) return PSIM_ERR_ARG;
+  if (!ctx->done) return PSIM_ERR_STATE;
+  *out = ctx->stats;
+  return PSIM_OK;
+}

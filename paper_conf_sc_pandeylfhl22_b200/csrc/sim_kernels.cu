@@ -1,0 +1,285 @@
+// sim_kernels.cu -- the integer side of the lockstep step (sm_100a):
+//   gather   (context construction, PAPER.md:93 steps 2.1-2.3, :123-127)
+//   update   (rounding + Clock advance + retire/compact/push, :99, :105-107)
+//   reduce   (per-sub-trace cycles -> local total, :107, :181)
+// One warp per sub-trace; state is structure-of-arrays in HBM (internal.h).
+//
+// Time features: every live entry satisfies retire > Clock (R4), and
+// retire - fetch = c + s <= 8190, so age = Clock - fetch < 8191 is computed
+// exactly from the low 32 bits of the clocks (q_fetch) whatever the absolute
+// Clock; the 65535 clamp of R7 is kept for completeness.
+#include "internal.h"
+
+namespace psim {
+
+__device__ __forceinline__ int lat_round(float y) {
+  // R7: nearest integer, ties to even, on the fp32 value; NaN -> 0; clamp [0, 4095]
+  if (isnan(y)) return 0;
+  float r = rintf(y);
+  if (r < 0.f) return 0;
+  if (r > (float)kLatMax) return kLatMax;
+  return (int)r;
+}
+
+template <typename T>
+__device__ __forceinline__ void store2(T* p, float a, float b);
+template <>
+__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
+  *reinterpret_cast<float2*>(p) = make_float2(a, b);
+}
+template <>
+__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);  // exact for |v| <= 256
+}
+
+// X[b][r][c]: row 0 = current instruction (time columns 0), rows 1..k = live
+// entries newest first (R6), rows > k zero (PAPER.md:93 zero padding).
+// Lane l writes columns 2l, 2l+1.
+template <typename T>
+__global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict__ x) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
+  const int c0 = 2 * lane, c1 = 2 * lane + 1;
+  for (uint64_t b = warp; b < a.n; b += nwarps) {
+    const int64_t ws = a.ws[b];
+    if (a.step >= a.e[b] - ws) continue;                      // sub-trace finished
+    const int64_t i = ws + a.step;
+    const int k = a.count[b];
+    const uint32_t clo = (uint32_t)a.clock[b];
+    T* xb = x + b * (uint64_t)(kRows * kFeatPad);
+    const uint32_t* qs = a.q_seq + b * kQStride;
+    const uint32_t* qf = a.q_fetch + b * kQStride;
+    const uint32_t* qc = a.q_cs + b * kQStride;
+    for (int r = 0; r < kRows; ++r) {
+      float v0 = 0.f, v1 = 0.f;
+      if (r <= k) {
+        int64_t row;
+        int age = 0, remc = 0, remr = 0;
+        if (r == 0) {
+          row = i;
+        } else {
+          const int ent = k - r;                                  // newest first
+          row = qs[ent];
+          const uint32_t cs = qc[ent];
+          const int c = cs & 0xFFFF, s = cs >> 16;
+          age = (int)(clo - qf[ent]);
+          remc = max(0, c - age);
+          remr = c + s - age;
+          age = min(age, kTimeMax); remc = min(remc, kTimeMax); remr = min(remr, kTimeMax);
+        }
+        const uint8_t* ar = a.trace + (row - a.row_lo) * a.stride;
+        auto col = [&](int c) -> float {
+          if (c < 3) return c == 0 ? (float)age : (c == 1 ? (float)remc : (float)remr);
+          if (c < kFeat) return (float)__ldg(ar + (c - 3));
+          return 0.f;
+        };
+        v0 = col(c0);
+        v1 = col(c1);
+      }
+      store2<T>(xb + r * kFeatPad + c0, v0, v1);
+    }
+  }
+}
+
+static int grid_for(uint64_t warps, int block = 256) {
+  uint64_t blocks = (warps * 32 + block - 1) / block;
+  if (blocks > 148ull * 64) blocks = 148ull * 64;
+  if (blocks < 1) blocks = 1;
+  return (int)blocks;
+}
+
+void launch_gather_f32(const GatherArgs& a, float* x, cudaStream_t st) {
+  gather_kernel<float><<<grid_for(a.n), 256, 0, st>>>(a, x);
+}
+void launch_gather_bf16(const GatherArgs& a, __nv_bfloat16* x, cudaStream_t st) {
+  gather_kernel<__nv_bfloat16><<<grid_for(a.n), 256, 0, st>>>(a, x);
+}
+
+// ---------------------------------------------------------------------------
+// update: round (R7), Clock += f, push, retire every entry with retire <= Clock
+// (PAPER.md:107), ROB-full stall if more than cap entries remain (R5),
+// boundary / cycles bookkeeping, per-row records (parity).
+// Lane l owns entries l, l+32, l+64, l+96 in registers; stable compaction by
+// ballot + popc keeps fetch order.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) update_kernel(UpdateArgs a) {
+  const int lane = threadIdx.x & 31;
+  const unsigned lt_mask = (1u << lane) - 1u;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
+  for (uint64_t b = warp; b < a.st.n; b += nwarps) {
+    const int64_t ws = a.st.ws[b], s_b = a.st.s[b], e_b = a.st.e[b];
+    const int64_t nsteps = e_b - ws;
+    if (a.step >= nsteps) continue;
+    const int64_t i = ws + a.step;
+    int f, c, s;
+    if (a.forced) {
+      const uint16_t* p = a.forced + (i - a.row_lo) * 3;
+      f = p[0]; c = p[1]; s = p[2];
+    } else {
+      f = lat_round(a.y[b * 3 + 0]);
+      c = lat_round(a.y[b * 3 + 1]);
+      s = lat_round(a.y[b * 3 + 2]);
+    }
+    int64_t clock = a.st.clock[b];
+    const int k = a.st.count[b];
+    uint32_t* qs = a.st.q_seq + b * kQStride;
+    uint32_t* qf = a.st.q_fetch + b * kQStride;
+    uint32_t* qc = a.st.q_cs + b * kQStride;
+
+    clock += f;
+    const uint32_t clo_push = (uint32_t)clock;
+    uint32_t eseq[4], efet[4], ecs[4];
+    bool valid[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const int ent = lane + 32 * m;
+      valid[m] = ent < k;
+      if (valid[m]) { eseq[m] = qs[ent]; efet[m] = qf[ent]; ecs[m] = qc[ent]; }
+      if (ent == k) {                                      // push the predicted instruction (R4)
+        valid[m] = true;
+        eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16);
+      }
+    }
+    __syncwarp();
+    // retire: keep iff retire > Clock  <=>  c + s - age > 0
+    auto live = [&](int m, uint32_t clo) -> bool {
+      if (!valid[m]) return false;
+      const int cs_sum = (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16);
+      return cs_sum - (int)(clo - efet[m]) > 0;
+    };
+    bool keep[4];
+    int kept = 0;
+    uint32_t clo = (uint32_t)clock;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
+    if (kept > a.cap) {                                    // ROB-full stall: Clock = min retire (R5)
+      int dmin = 0x7fffffff;
+#pragma unroll
+      for (int m = 0; m < 4; ++m)
+        if (keep[m]) dmin = min(dmin, (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16) - (int)(clo - efet[m]));
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) dmin = min(dmin, __shfl_xor_sync(0xffffffffu, dmin, o));
+      clock += dmin;
+      clo = (uint32_t)clock;
+      kept = 0;
+#pragma unroll
+      for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
+      if (lane == 0) atomicAdd(a.st.stalls, 1ull);
+    }
+    int base = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const unsigned bal = __ballot_sync(0xffffffffu, keep[m]);
+      if (keep[m]) {
+        const int pos = base + __popc(bal & lt_mask);
+        qs[pos] = eseq[m]; qf[pos] = efet[m]; qc[pos] = ecs[m];
+      }
+      base += __popc(bal);
+    }
+    if (lane == 0) {
+      a.st.count[b] = base;
+      a.st.clock[b] = clock;
+      int64_t bnd = a.st.bnd[b];
+      if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
+      if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
+      atomicAdd(a.st.k_hist + k, 1ull);
+      if (i >= s_b) {
+        const int64_t r = i - a.row_lo;
+        if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)f; a.rec_lat[3 * r + 1] = (uint16_t)c; a.rec_lat[3 * r + 2] = (uint16_t)s; }
+        if (a.rec_k) a.rec_k[r] = k;
+        if (a.rec_clock) a.rec_clock[r] = clock;
+      }
+    }
+  }
+}
+
+void launch_update(const UpdateArgs& a, cudaStream_t st) {
+  update_kernel<<<grid_for(a.st.n), 256, 0, st>>>(a);
+}
+
+__global__ void state_init_kernel(SimState s) {
+  const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (t < s.n) { s.clock[t] = 0; s.bnd[t] = 0; s.cycles[t] = 0; s.count[t] = 0; }
+  if (t < 112) s.k_hist[t] = 0;
+  if (t == 0) { *s.stalls = 0; *s.total = 0; }
+}
+void launch_state_init(const SimState& s, cudaStream_t st) {
+  uint64_t n = s.n > 112 ? s.n : 112;
+  state_init_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(s);
+}
+
+// total = sum_j cycles_j (int64, exact and order independent)
+__global__ void __launch_bounds__(1024) reduce_kernel(SimState s) {
+  long long acc = 0;
+  for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < s.n; t += (uint64_t)gridDim.x * blockDim.x)
+    acc += s.cycles[t];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  __shared__ long long part[32];
+  if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    acc = threadIdx.x < (blockDim.x >> 5) ? part[threadIdx.x] : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (threadIdx.x == 0) atomicAdd((unsigned long long*)s.total, (unsigned long long)acc);
+  }
+}
+void launch_reduce_cycles(const SimState& s, cudaStream_t st) {
+  unsigned blocks = (unsigned)((s.n + 1023) / 1024);
+  if (blocks > 148) blocks = 148;
+  if (blocks < 1) blocks = 1;
+  reduce_kernel<<<blocks, 1024, 0, st>>>(s);
+}
+
+// head (fc2, fp32 on CUDA cores): y[b][o] = b[o] + sum_i h[b][i] w[o][i]
+__global__ void __launch_bounds__(256) head_kernel(const float* __restrict__ h, const float* __restrict__ w,
+                                                   const float* __restrict__ bias, int in,
+                                                   float* __restrict__ y, uint64_t n) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
+  for (uint64_t b = warp; b < n; b += nwarps) {
+    float a0 = 0.f, a1 = 0.f, a2 = 0.f;
+    for (int t = lane; t < in; t += 32) {
+      const float v = h[b * in + t];
+      a0 = fmaf(v, __ldg(w + t), a0);
+      a1 = fmaf(v, __ldg(w + in + t), a1);
+      a2 = fmaf(v, __ldg(w + 2 * in + t), a2);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      a0 += __shfl_xor_sync(0xffffffffu, a0, o);
+      a1 += __shfl_xor_sync(0xffffffffu, a1, o);
+      a2 += __shfl_xor_sync(0xffffffffu, a2, o);
+    }
+    if (lane == 0) {
+      y[b * 3 + 0] = a0 + bias[0];
+      y[b * 3 + 1] = a1 + bias[1];
+      y[b * 3 + 2] = a2 + bias[2];
+    }
+  }
+}
+void launch_head(const float* h, const float* w, const float* b, int in, float* y, uint64_t n,
+                 cudaStream_t st) {
+  head_kernel<<<grid_for(n), 256, 0, st>>>(h, w, b, in, y, n);
+}
+
+__global__ void pad_inputs_kernel(const float* __restrict__ X, uint64_t B, void* x, bool bf16) {
+  const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const uint64_t total = B * kRows * kFeatPad;
+  if (t >= total) return;
+  const int c = (int)(t % kFeatPad);
+  const uint64_t br = t / kFeatPad;
+  const float v = c < kFeat ? X[br * kFeat + c] : 0.f;
+  if (bf16) reinterpret_cast<__nv_bfloat16*>(x)[t] = __float2bfloat16_rn(v);
+  else reinterpret_cast<float*>(x)[t] = v;
+}
+void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st) {
+  const uint64_t total = B * kRows * kFeatPad;
+  pad_inputs_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(X, B, x, bf16);
+}
+
+}  // namespace psim
