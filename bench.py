@@ -1,0 +1,328 @@
+"""bench.py -- parallel sub-trace ML simulation throughput on B200 (MIPS).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl psim|reference] [--config c3|c2|c1]
+
+A step is one pass of the whole hot path -- psim_simulate: every lockstep step
+of gather -> CNN GEMMs -> head -> round/update over all sub-traces, then the
+cycle reduction (+ NCCL all-reduce for N > 1) -- over one synthetic trace.
+Default workload: BASELINE.json configs[2] (the metric's config): a
+100M-instruction SPEC-like synthetic trace, 65536 sub-traces, W = 110
+(= Context_length), C3 CNN, bf16 operands; it fits one GPU.
+
+value  = instructions simulated by all ranks (warm-up excluded) / max-over-ranks
+         device time of K steps, trace resident in HBM before the timed region.
+e2e    = the same through psim_load_trace with a PINNED HOST trace: the H2D copy
+         of each rank's rows and the D2H of the total are inside every step.
+roofline / cpu_baseline / clocks: see DESIGN.md "measurement".
+
+Under torchrun (N > 1) each rank owns the contiguous sub-trace block
+[g N/G, (g+1) N/G) and generates only its own trace rows (counter-based
+generator), so nothing but the final int64 cycle count crosses NVLink.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import signal
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    "c1": dict(L=10_000, N=1, W=0, arch="M2", precision="fp32", seed_off=0,
+               desc="config1: 10k-instruction synthetic trace, 1 sub-trace, queue 111, M2 CNN, fp32"),
+    "c2": dict(L=1_000_000, N=1024, W=1000, arch="C3", precision="bf16", seed_off=1,
+               desc="config2: 1M-instruction synthetic SPEC-like trace, 1024 sub-traces, W=1000, C3 CNN, bf16"),
+    "c3": dict(L=100_000_000, N=65536, W=110, arch="C3", precision="bf16", seed_off=2,
+               desc="config3: 100M-instruction synthetic SPEC-like trace, 65536 sub-traces, W=110, C3 CNN, bf16"),
+}
+METRIC = "simulated instr/sec (MIPS, 8×B200 device-timed) + cycle error vs CPU oracle"
+REASONS = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# --------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi sampling DURING the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = "index,clocks.sm,clocks.max.sm,power.draw," + ",".join(f"clocks_event_reasons.{r}" for r in REASONS)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL, start_new_session=True)
+        except FileNotFoundError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        os.killpg(self.p.pid, signal.SIGTERM)
+        self.p.wait()
+        self.f.flush()
+        rows = [l.split(",") for l in open(self.f.name).read().strip().splitlines() if l.strip()]
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].strip().replace(".", "").isdigit()]
+        reasons = sorted({REASONS[i] for r in rows for i in range(len(REASONS))
+                          if len(r) > 4 + i and "Active" in r[4 + i] and "Not" not in r[4 + i]})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+# --------------------------------------------------------------------------- roofline
+def roofline(stats, k_steps, cfg):
+    """Dominant kernel class by device time; algorithmic work per launch / average
+    launch duration (CUDA events on the launch stream, PSIM_PROFILE)."""
+    names, ms, launches = stats["kernel_names"], stats["kernel_ms"], stats["kernel_launches"]
+    total_ms = sum(ms)
+    dom = int(np.argmax(ms))
+    pk, src = peaks()
+    out = {"kernel": names[dom], "share": round(ms[dom] / total_ms, 4) if total_ms else None}
+    avg_s = ms[dom] / 1e3 / max(launches[dom], 1)
+    hist = np.array(stats["k_hist"], np.float64)
+    kmean = float((hist * np.arange(112)).sum() / max(hist.sum(), 1))
+    if names[dom].startswith("gemm_layer"):
+        li = int(names[dom][-1])
+        M, N, K = stats["layer_m"][li], stats["layer_n"][li], stats["layer_k"][li]
+        k_alg = 100 if li == 0 else K          # conv1: 2 rows x 50 real features (features padded to 64)
+        flops = 2.0 * M * N * k_alg
+        achieved = flops / avg_s / 1e12
+        peak = pk["bf16_tflops_sustained"] if cfg["precision"] == "bf16" else 74.0
+        out.update(bound="tensor", achieved=round(achieved, 2), peak=peak, unit="TFLOP/s",
+                   frac=round(achieved / peak, 4), flops_per_launch=flops,
+                   peak_source=(src + " bf16 sustained") if cfg["precision"] == "bf16" else "derived fp32 SIMT")
+    else:
+        n = stats["subtraces"]
+        if names[dom] == "gather":   # X write (bf16 112x64) + trace rows (k+1)x48 + queue (k x 12 B)
+            byts = n * (112 * 64 * 2 + (kmean + 1) * 48 + kmean * 12)
+        else:                        # update: queue read+write (2 x k x 12 B) + state + y
+            byts = n * (2 * (kmean + 1) * 12 + 64)
+        achieved = byts / avg_s / 1e9
+        out.update(bound="hbm", achieved=round(achieved, 1), peak=pk["hbm_gbs"], unit="GB/s",
+                   frac=round(achieved / pk["hbm_gbs"], 4), bytes_per_launch=byts, peak_source=src + " hbm")
+    out["traffic"] = ncu_traffic(names[dom])
+    out["avg_launch_us"] = round(avg_s * 1e6, 2)
+    out["kernels"] = {names[i]: {"ms": round(ms[i] / k_steps, 3), "launches": launches[i] // k_steps,
+                                 "share": round(ms[i] / total_ms, 4) if total_ms else None}
+                      for i in range(len(names)) if launches[i]}
+    out["k_mean"] = round(kmean, 2)
+    return out
+
+
+def ncu_traffic(kernel_class):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        v = d.get(kernel_class)
+        return v.get("dram_bytes_per_launch") if isinstance(v, dict) else v
+    return None
+
+
+# --------------------------------------------------------------------------- CPU oracle
+def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None):
+    """Run the oracle (as it stands, single thread) on whole sub-traces of the same
+    workload until ~budget_s of CPU time; returns (instructions, seconds, cycles)."""
+    import oracle
+    import synth
+    w = synth.weights(cfg["arch"])
+    mode = oracle.BF16 if cfg["precision"] == "bf16" else oracle.FP64
+    rng = np.random.default_rng(7)
+    done, t_used, per = 0, 0.0, {}
+    js = list(j_list) if j_list is not None else []
+    while True:
+        if j_list is None:
+            j = int(rng.integers(0, N))
+        else:
+            if not js:
+                break
+            j = js.pop(0)
+        s, e = j * L // N, (j + 1) * L // N
+        ws = max(0, s - W)
+        if tr_rows is not None and ws >= row_lo and e - row_lo <= tr_rows.shape[0]:
+            sl = tr_rows[ws - row_lo:e - row_lo]
+        else:
+            sl = synth.trace(e - ws, synth.TRACE_SEED_BASE + cfg["seed_off"], r0=ws)
+        t0 = time.perf_counter()
+        r = oracle.simulate(sl, N, W, arch=cfg["arch"], weights=w, mode=mode, j0=j, nj=1, L=L, row_offset=ws,
+                            want_rows=False)
+        t_used += time.perf_counter() - t0
+        done += e - s
+        per[j] = int(r["cycles"][0])
+        if j_list is None and t_used >= budget_s:
+            break
+    return done, t_used, per
+
+
+# --------------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="psim", choices=["psim", "reference"])
+    ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    cfg = CONFIGS[args.config]
+    L, N, W = cfg["L"], cfg["N"], cfg["W"]
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    config = {"workload": cfg["desc"], "instructions": L, "subtraces": N, "warmup_W": W, "cnn": cfg["arch"],
+              "queue_rows": 111, "precision": cfg["precision"],
+              "l2": "inputs larger than L2 (trace %.1f GB resident in HBM)" % (L * 48 / 1e9)}
+
+    if args.impl == "reference":
+        # the oracle as it stands, on rank 0 only, on the host cores
+        if rank != 0:
+            return
+        import synth  # noqa: F401
+        per_step = max(2.0, args.cpu_budget / 3)
+        times, insts = [], 0
+        for it in range(args.warmup + args.steps):
+            n_i, t, _ = oracle_sample(cfg, None, 0, per_step, L, N, W)
+            if it >= args.warmup:
+                times.append(t); insts += n_i
+        tot = sum(times)
+        val = insts / tot / 1e6
+        line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "MIPS", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64" if cfg["precision"] == "fp32" else "f64 (bf16 operand rounding)",
+                "data": "synthetic", "config": config,
+                "cpu_baseline": {"value": val, "unit": "MIPS", "cores": 1, "kind": "oracle",
+                                 "sample": f"{insts} instructions of whole random sub-traces of {args.config} per "
+                                           f"{args.steps} steps, single-threaded plain-C oracle"},
+                "e2e": {"value": val, "unit": "MIPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_pandeylfhl22_b200 as P
+    import synth
+
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    nccl_id = None
+    if world > 1:
+        obj = [P.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+
+    rr = P.partition_range(L, N, W, rank, world)
+    rows = rr.row_hi - rr.row_lo
+    t0 = time.time()
+    host = torch.empty((rows, 48), dtype=torch.uint8, pin_memory=True)
+    synth.trace_into(host.numpy(), synth.TRACE_SEED_BASE + cfg["seed_off"], rr.row_lo)
+    dev = host.cuda()
+    w = synth.weights(cfg["arch"])
+    log(f"[rank {rank}] trace rows [{rr.row_lo},{rr.row_hi}) generated in {time.time() - t0:.1f}s")
+
+    stream = torch.cuda.Stream()
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=rank, world_size=world, nccl_id=nccl_id,
+                      stream=stream.cuda_stream, profile=True)
+    sim.load_model(cfg["arch"], w)
+
+    def timed(trace_tensor, k_steps, warm):
+        sim.load_trace(trace_tensor, n_instr=L, first_row=rr.row_lo)
+        sim.partition(N, W)
+        for _ in range(warm):
+            sim.simulate()
+        barrier()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        clk = ClockSampler(local_rank)
+        ev0.record(stream)
+        tot = None
+        kms = None
+        for _ in range(k_steps):
+            sim.simulate()
+            tot = sim.total_cycles()            # D2H of the step's result
+            st = sim.stats()
+            kms = st if kms is None else {**st, "kernel_ms": [a + b for a, b in zip(kms["kernel_ms"], st["kernel_ms"])],
+                                          "kernel_launches": [a + b for a, b in zip(kms["kernel_launches"], st["kernel_launches"])]}
+        ev1.record(stream)
+        barrier()
+        clocks = clk.stop()
+        ms = ev0.elapsed_time(ev1)
+        return max_over_ranks(ms), tot, kms, clocks
+
+    ms, total, stats, clocks = timed(dev, args.steps, args.warmup)
+    value = L * args.steps / (ms / 1e3) / 1e6
+    e2e = None
+    if not args.no_e2e:
+        ms_e, total_e, st_e, _ = timed(host, args.steps, 1)
+        assert total_e == total, (total_e, total)
+        ranges = [P.partition_range(L, N, W, g, world) for g in range(world)]
+        e2e = {"value": L * args.steps / (ms_e / 1e3) / 1e6, "unit": "MIPS",
+               "h2d_bytes_per_step": int(sum((x.row_hi - x.row_lo) * 48 for x in ranges)),
+               "d2h_bytes_per_step": 8 * world}
+
+    line = {"metric": METRIC, "value": value, "unit": "MIPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": cfg["precision"], "data": "synthetic", "config": config,
+            "total_cycles": total, "e2e": e2e, "gpu_launches": int(sum(stats["kernel_launches"])),
+            "clocks": clocks}
+    if rank == 0:
+        line["roofline"] = roofline(stats, args.steps, cfg)
+        line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces")}
+        line["warmup_overhead"] = round(stats["simulated"] / stats["counted"] - 1, 4)
+    if rank == 0 and world == 1:
+        # cpu_baseline: the oracle as it stands on a bounded sample of the same workload,
+        # plus the sampled sub-traces' cycles vs the GPU (parity sample)
+        n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W)
+        gcyc = sim.subtrace_cycles()
+        errs = [abs(int(gcyc[j]) - c) / max(c, 1) for j, c in per.items()]
+        line["cpu_baseline"] = {"value": n_i / t / 1e6, "unit": "MIPS", "cores": 1, "kind": "oracle",
+                                "sample": f"{len(per)} whole sub-traces ({n_i} counted instructions, W={W} warm-up "
+                                          f"each) of {args.config}, plain-C oracle "
+                                          f"{'bf16-operand' if cfg['precision'] == 'bf16' else 'fp64'} mode, 1 thread"}
+        line["parity_sample"] = {"subtraces": sorted(per), "max_rel_cycle_err": max(errs) if errs else None}
+    sim.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -52,6 +52,20 @@ extern "C" {
 /* flags for psim_opts.flags */
 #define PSIM_RECORD_ROWS 1u  /* keep per-instruction (f,c,s), context count k and Clock
                                 (device buffers sized to the rank's rows) for parity reads */
+#define PSIM_FORCE_PREDICT 4u /* with psim_force_latencies: still run gather + CNN + rounding every
+                                step and record the CNN's (f,c,s) in the per-row outputs, while the
+                                queue update follows the forced latencies (decision parity on a
+                                given trajectory, R17)                              */
+#define PSIM_PROFILE 2u      /* time every kernel class with CUDA events on the launch stream
+                                (psim_stats.kernel_ms / kernel_launches)                    */
+
+/* kernel classes reported in psim_stats.kernel_ms (names: psim_kernel_class_name) */
+#define PSIM_KC_GATHER 0
+#define PSIM_KC_LAYER0 1   /* first GEMM layer (conv1); layer i is PSIM_KC_LAYER0 + i */
+#define PSIM_KC_HEAD 5
+#define PSIM_KC_UPDATE 6
+#define PSIM_KC_OTHER 7
+#define PSIM_KC_COUNT 8
 
 typedef struct psim_ctx psim_ctx;  /* opaque; owns every device allocation it makes */
 
@@ -89,6 +103,10 @@ typedef struct {
     int64_t local_cycles;     /* sum of this rank's sub-trace cycles                       */
     int32_t trace_mode;       /* 0 device-resident, 1 pinned host (zero-copy loader), 2 pageable */
     int32_t pad;
+    double kernel_ms[8];      /* PSIM_PROFILE: summed device time per kernel class          */
+    uint64_t kernel_launches[8]; /* launches per kernel class                               */
+    uint64_t layer_m[4];      /* GEMM rows per launch of layers 0..3 (M = sub-traces x positions) */
+    uint32_t layer_n[4], layer_k[4];  /* GEMM N and K of layers 0..3 (device shapes)        */
 } psim_stats;
 
 /* Create a context on opts->device.  world_size > 1 with nccl_id != NULL
@@ -175,6 +193,14 @@ int psim_get_stats(const psim_ctx* ctx, psim_stats* out);
  * fp32 (the instruction-major input of PAPER.md:93), Y host [B][3] fp32 raw
  * outputs before rounding.  Runs the same kernels as simulate. */
 int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float* Y);
+
+/* Name of kernel class i (0 <= i < PSIM_KC_COUNT), or NULL. */
+const char* psim_kernel_class_name(int i);
+
+/* Fill out[128] with a fresh ncclUniqueId (call on rank 0, broadcast the bytes
+ * to the other ranks, pass them as psim_opts.nccl_id).  PSIM_ERR_NCCL if NCCL
+ * cannot be loaded. */
+int psim_nccl_unique_id(void* out128);
 
 /* Library build string (compiler, arch, kernels). */
 const char* psim_version(void);

@@ -152,13 +152,15 @@ def partition(L: int, N: int, W: int):
 
 def simulate(trace: np.ndarray, N: int, W: int, *, arch: str = "C3", weights=None,
              mode: int = FP64, cap: int = 110, forced_lat=None, j0: int = 0, nj=None,
-             clock0: int = 0, want_rows: bool = True):
+             clock0: int = 0, want_rows: bool = True, L: int | None = None, row_offset: int = 0):
     """Simulate sub-traces [j0, j0+nj) of the N-way partition.
 
-    Returns dict(cycles, boundary, total, stalls, and per-row lat/y/k/clock if want_rows).
+    ``trace`` holds rows [row_offset, row_offset + len(trace)) of an L-row trace
+    (default: the whole trace).  Returns dict(cycles, boundary, total, stalls,
+    and per-row lat/y/k/clock over all L rows if want_rows).
     """
     trace = np.ascontiguousarray(trace, dtype=np.uint8)
-    L = trace.shape[0]
+    L = trace.shape[0] + row_offset if L is None else L
     nj = N - j0 if nj is None else nj
     w = None if weights is None else np.ascontiguousarray(weights, dtype=np.float32)
     forced = None if forced_lat is None else np.ascontiguousarray(forced_lat, dtype=np.uint16)
@@ -173,7 +175,7 @@ def simulate(trace: np.ndarray, N: int, W: int, *, arch: str = "C3", weights=Non
     stalls = ctypes.c_int64(0)
     rc = lib().oracle_simulate(
         ARCH.get(arch, 0), mode, _ptr(w), 0 if w is None else w.size,
-        _ptr(trace), trace.shape[1], L, N, W, cap,
+        ctypes.c_void_p(trace.ctypes.data - row_offset * trace.shape[1]), trace.shape[1], L, N, W, cap,
         _ptr(forced), j0, nj, clock0,
         _ptr(cycles), _ptr(boundary), _ptr(lat), _ptr(y), _ptr(k), _ptr(clk), ctypes.byref(stalls))
     if rc != 0:

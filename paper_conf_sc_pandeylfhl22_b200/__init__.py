@@ -23,6 +23,8 @@ OK, ERR_ARG, ERR_STATE, ERR_CUDA, ERR_NCCL, ERR_OOM, ERR_UNSUPPORTED = 0, -1, -2
 FP32, BF16 = 0, 1
 ARCH = {"M2": 1, "C3": 2, "RB7": 3}
 RECORD_ROWS = 1
+PROFILE = 2
+FORCE_PREDICT = 4
 MAX_CAP = 110
 NATTR = 47
 
@@ -49,18 +51,21 @@ class Stats(ctypes.Structure):
                 ("simulated", ctypes.c_uint64), ("counted", ctypes.c_uint64), ("subtraces", ctypes.c_uint64),
                 ("h2d_bytes", ctypes.c_uint64), ("gpu_launches", ctypes.c_uint64), ("sim_ms", ctypes.c_double),
                 ("load_ms", ctypes.c_double), ("local_cycles", ctypes.c_int64), ("trace_mode", ctypes.c_int32),
-                ("pad", ctypes.c_int32)]
+                ("pad", ctypes.c_int32), ("kernel_ms", ctypes.c_double * 8), ("kernel_launches", ctypes.c_uint64 * 8),
+                ("layer_m", ctypes.c_uint64 * 4), ("layer_n", ctypes.c_uint32 * 4), ("layer_k", ctypes.c_uint32 * 4)]
 
     def as_dict(self):
-        d = {f: getattr(self, f) for f, _ in self._fields_ if f not in ("k_hist", "pad")}
-        d["k_hist"] = list(self.k_hist)
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "pad"}
+        for f in ("k_hist", "kernel_ms", "kernel_launches", "layer_m", "layer_n", "layer_k"):
+            d[f] = list(d[f])
+        d["kernel_names"] = [lib().psim_kernel_class_name(i).decode() for i in range(8)]
         return d
 
 
 EXPORTS = ["psim_create", "psim_destroy", "psim_load_trace", "psim_partition", "psim_load_model",
            "psim_simulate", "psim_total_cycles", "psim_last_error", "psim_force_latencies", "psim_get_rows",
            "psim_get_subtrace_cycles", "psim_rank_range", "psim_get_stats", "psim_cnn_forward", "psim_version",
-           "psim_partition_range"]
+           "psim_partition_range", "psim_kernel_class_name", "psim_nccl_unique_id"]
 
 _lib = None
 
@@ -93,6 +98,9 @@ def lib():
         L.psim_cnn_forward.argtypes = [P, P, c.c_uint64, P]
         L.psim_version.restype = c.c_char_p
         U = c.POINTER(c.c_uint64)
+        L.psim_kernel_class_name.argtypes = [c.c_int]
+        L.psim_kernel_class_name.restype = c.c_char_p
+        L.psim_nccl_unique_id.argtypes = [P]
         L.psim_partition_range.argtypes = [c.c_uint64, c.c_uint64, c.c_uint64, c.c_int, c.c_int, U, U, U, U, U]
         _lib = L
     return _lib
@@ -129,6 +137,15 @@ def partition_range(L: int, N: int, W: int, rank: int = 0, world_size: int = 1) 
     return RankRange(*[int(x.value) for x in v])
 
 
+def nccl_unique_id() -> bytes:
+    """128-byte ncclUniqueId (rank 0), to broadcast with torch.distributed."""
+    buf = ctypes.create_string_buffer(128)
+    rc = lib().psim_nccl_unique_id(buf)
+    if rc != OK:
+        raise PsimError(rc, "NCCL unavailable")
+    return buf.raw
+
+
 def all_reduce_total(local_total: int, group=None) -> int:
     """Sum per-rank totals over a torch.distributed group (used when the context
     was created without an NCCL id, e.g. gloo on CPU)."""
@@ -144,7 +161,8 @@ class Simulator:
 
     def __init__(self, device: int = 0, precision: str = "bf16", queue_cap: int = MAX_CAP,
                  rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
-                 stream=None, record_rows: bool = False, chunk_steps: int = 0):
+                 stream=None, record_rows: bool = False, chunk_steps: int = 0, profile: bool = False,
+                 force_predict: bool = False):
         self._keep = []
         idbuf = None
         if nccl_id is not None:
@@ -155,7 +173,8 @@ class Simulator:
                   queue_cap=queue_cap, precision=BF16 if precision == "bf16" else FP32,
                   chunk_steps=chunk_steps,
                   stream=ctypes.c_void_p(int(stream)) if stream is not None else None,
-                  flags=RECORD_ROWS if record_rows else 0)
+                  flags=(RECORD_ROWS if record_rows else 0) | (PROFILE if profile else 0)
+                  | (FORCE_PREDICT if force_predict else 0))
         h = ctypes.c_void_p()
         rc = lib().psim_create(ctypes.byref(o), ctypes.byref(h))
         if rc != OK:

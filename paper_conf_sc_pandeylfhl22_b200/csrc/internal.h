@@ -93,7 +93,7 @@ struct UpdateArgs {
   int64_t row_lo;
   int64_t step;
   int cap;
-  const float* y;            // [n][3] raw CNN outputs (CNN mode) or nullptr
+  const float* y;            // [n][3] raw CNN outputs (CNN mode, or forced+predict) or nullptr
   const uint16_t* forced;    // [rows][3] teacher-forced latencies (row - row_lo) or nullptr
   uint16_t* rec_lat;         // [rows][3] or nullptr (PSIM_RECORD_ROWS)
   int32_t* rec_k;            // [rows] or nullptr

@@ -28,6 +28,7 @@ struct NcclApi {
   ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
   const char* (*errStr)(ncclResult_t) = nullptr;
+  ncclResult_t (*getUniqueId)(ncclUniqueId*) = nullptr;
 };
 NcclApi g_nccl;
 std::mutex g_nccl_mu;
@@ -44,7 +45,8 @@ bool load_nccl() {
   g_nccl.allReduce = (decltype(g_nccl.allReduce))dlsym(h, "ncclAllReduce");
   g_nccl.commDestroy = (decltype(g_nccl.commDestroy))dlsym(h, "ncclCommDestroy");
   g_nccl.errStr = (decltype(g_nccl.errStr))dlsym(h, "ncclGetErrorString");
-  g_nccl.ok = g_nccl.commInitRank && g_nccl.allReduce && g_nccl.commDestroy && g_nccl.errStr;
+  g_nccl.getUniqueId = (decltype(g_nccl.getUniqueId))dlsym(h, "ncclGetUniqueId");
+  g_nccl.ok = g_nccl.commInitRank && g_nccl.allReduce && g_nccl.commDestroy && g_nccl.errStr && g_nccl.getUniqueId;
   return g_nccl.ok;
 }
 
@@ -57,8 +59,49 @@ inline uint16_t f32_to_bf16_rne(float f) {
 }
 }  // namespace
 
+// Per-kernel-class device timing with CUDA events on the launch stream
+// (PSIM_PROFILE); launch counting is always on (psim_stats.gpu_launches).
+struct Prof {
+  bool on = false;
+  cudaStream_t st = nullptr;
+  std::vector<cudaEvent_t> pool;
+  size_t used = 0;
+  std::vector<std::pair<int, size_t>> marks;   // (class, index of the start event)
+  size_t open_idx = 0;
+  uint64_t launches[PSIM_KC_COUNT] = {};
+  void reset(bool enable, cudaStream_t s) {
+    on = enable; st = s; used = 0; marks.clear();
+    for (auto& l : launches) l = 0;
+  }
+  cudaEvent_t next() {
+    if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
+    return pool[used++];
+  }
+  void begin(int cls) {
+    launches[cls]++;
+    if (!on) return;
+    open_idx = used;
+    cudaEventRecord(next(), st);
+  }
+  void end(int cls) {
+    if (!on) return;
+    cudaEventRecord(next(), st);
+    marks.push_back({cls, open_idx});
+  }
+  void collect(double* ms) {
+    for (int c = 0; c < PSIM_KC_COUNT; ++c) ms[c] = 0;
+    for (auto& m : marks) {
+      float t = 0;
+      cudaEventElapsedTime(&t, pool[m.second], pool[m.second + 1]);
+      ms[m.first] += t;
+    }
+  }
+  ~Prof() { for (auto e : pool) cudaEventDestroy(e); }
+};
+
 struct psim_ctx {
   psim_opts opts{};
+  Prof prof;
   int cap = 110;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -388,8 +431,9 @@ static int ensure_buffers(psim_ctx* ctx, uint64_t n) {
 }
 
 // Run the lowered CNN on buf.x (n items) -> buf.y.  Counts launches.
-static int run_cnn(psim_ctx* ctx, uint64_t n, uint64_t* launches) {
+static int run_cnn(psim_ctx* ctx, uint64_t n) {
   const Model& m = ctx->model;
+  Prof& pf = ctx->prof;
   const bool bf16 = m.precision == PSIM_BF16;
   const void* in = ctx->buf.x;
   for (size_t li = 0; li < m.layers.size(); ++li) {
@@ -397,17 +441,19 @@ static int run_cnn(psim_ctx* ctx, uint64_t n, uint64_t* launches) {
     const bool last = li + 1 == m.layers.size();
     void* out = last ? (void*)ctx->buf.h : ctx->buf.act[li];
     const int64_t M = (int64_t)n * g.rows_per_item;
+    pf.begin(PSIM_KC_LAYER0 + (int)li);
     if (bf16) {
       if (g.w_tc) launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
       else launch_gemm_simt_bf16((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
     } else {
       launch_gemm_simt_f32((const float*)in, (const float*)g.w, g.bias, (float*)out, M, g.N, g.K, g.relu, ctx->stream);
     }
-    (*launches)++;
+    pf.end(PSIM_KC_LAYER0 + (int)li);
     in = out;
   }
+  pf.begin(PSIM_KC_HEAD);
   launch_head(ctx->buf.h, m.head_w, m.head_b, m.head_in, ctx->buf.y, n, ctx->stream);
-  (*launches)++;
+  pf.end(PSIM_KC_HEAD);
   return PSIM_OK;
 }
 
@@ -422,8 +468,8 @@ extern "C" int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float
   cudaError_t e = cudaMemcpyAsync(dX, X, B * kRows * kFeat * sizeof(float), cudaMemcpyHostToDevice, ctx->stream);
   if (e == cudaSuccess) {
     launch_pad_inputs(dX, B, ctx->buf.x, ctx->model.precision == PSIM_BF16, ctx->stream);
-    uint64_t l = 0;
-    run_cnn(ctx, B, &l);
+    ctx->prof.reset(false, ctx->stream);
+    run_cnn(ctx, B);
     e = cudaMemcpyAsync(Y, ctx->buf.y, B * 3 * sizeof(float), cudaMemcpyDeviceToHost, ctx->stream);
   }
   if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
@@ -467,18 +513,21 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   if (!ctx->have_trace || !ctx->partitioned) FAIL(PSIM_ERR_STATE, "simulate needs load_trace and partition");
   const bool forced = !ctx->forced.empty();
   if (!forced && !ctx->model.loaded) FAIL(PSIM_ERR_STATE, "simulate needs load_model or force_latencies");
+  const bool predict = !forced || (ctx->opts.flags & PSIM_FORCE_PREDICT);   // run the CNN each step
+  if (predict && !ctx->model.loaded) FAIL(PSIM_ERR_STATE, "PSIM_FORCE_PREDICT needs load_model");
   CK(cudaSetDevice(ctx->opts.device));
   cudaStream_t st = ctx->stream;
   const uint64_t n = ctx->j1 - ctx->j0;
   const int64_t rows = ctx->row_hi - ctx->row_lo;
-  uint64_t launches = 0;
   psim_stats stats{};
+  Prof& pf = ctx->prof;
+  pf.reset((ctx->opts.flags & PSIM_PROFILE) != 0, st);
   stats.subtraces = n;
   stats.trace_mode = ctx->trace_mode;
 
   int rc = ensure_state(ctx);
   if (rc) return rc;
-  if (!forced) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
+  if (predict) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
   const bool rec = (ctx->opts.flags & PSIM_RECORD_ROWS) != 0;
   if (rec && ctx->rec_cap < (size_t)rows) {
     dfree(ctx->rec_lat); dfree(ctx->rec_k); dfree(ctx->rec_clock);
@@ -517,29 +566,33 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   }
   CK(cudaEventRecord(ctx->ev[1], st));
 
+  pf.begin(PSIM_KC_OTHER);
   launch_state_init(ctx->st, st);
-  launches++;
+  pf.end(PSIM_KC_OTHER);
   const bool bf16 = ctx->model.precision == PSIM_BF16;
   GatherArgs ga{dtr, ctx->row_lo, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e, ctx->st.clock, ctx->st.count,
                 ctx->st.q_seq, ctx->st.q_fetch, ctx->st.q_cs, n, 0};
-  UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, forced ? nullptr : ctx->buf.y,
+  UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
   for (int64_t t = 0; t < ctx->steps && n; ++t) {
-    if (!forced) {
+    if (predict) {
       ga.step = t;
+      pf.begin(PSIM_KC_GATHER);
       if (bf16) launch_gather_bf16(ga, (__nv_bfloat16*)ctx->buf.x, st);
       else launch_gather_f32(ga, (float*)ctx->buf.x, st);
-      launches++;
-      rc = run_cnn(ctx, n, &launches);
+      pf.end(PSIM_KC_GATHER);
+      rc = run_cnn(ctx, n);
       if (rc) return rc;
     }
     ua.step = t;
+    pf.begin(PSIM_KC_UPDATE);
     launch_update(ua, st);
-    launches++;
+    pf.end(PSIM_KC_UPDATE);
   }
+  pf.begin(PSIM_KC_OTHER);
   launch_reduce_cycles(ctx->st, st);
-  launches++;
+  pf.end(PSIM_KC_OTHER);
   CK(cudaGetLastError());
   if (ctx->comm) {
     ncclResult_t r = g_nccl.allReduce(ctx->st.total, ctx->st.total, 1, ncclInt64, ncclSum, ctx->comm, st);
@@ -564,7 +617,16 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   for (uint64_t b = 0; b < n; ++b) { sim += ctx->h_e[b] - ctx->h_ws[b]; cnt += ctx->h_e[b] - ctx->h_s[b]; }
   stats.simulated = sim;
   stats.counted = cnt;
+  uint64_t launches = 0;
+  for (int c = 0; c < PSIM_KC_COUNT; ++c) { stats.kernel_launches[c] = pf.launches[c]; launches += pf.launches[c]; }
   stats.gpu_launches = launches;
+  pf.collect(stats.kernel_ms);
+  for (size_t li = 0; li < ctx->model.layers.size() && li < 4 && predict; ++li) {
+    const GemmLayer& g = ctx->model.layers[li];
+    stats.layer_m[li] = n * g.rows_per_item;
+    stats.layer_n[li] = g.N;
+    stats.layer_k[li] = g.K;
+  }
   stats.sim_ms = ms_all;
   stats.load_ms = ms_load;
   if (ctx->comm == nullptr) stats.local_cycles = total;
@@ -578,6 +640,21 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   }
   ctx->stats = stats;
   ctx->done = true;
+  return PSIM_OK;
+}
+
+extern "C" const char* psim_kernel_class_name(int i) {
+  static const char* names[PSIM_KC_COUNT] = {"gather", "gemm_layer0", "gemm_layer1", "gemm_layer2",
+                                             "gemm_layer3", "head", "update", "other"};
+  return (i >= 0 && i < PSIM_KC_COUNT) ? names[i] : nullptr;
+}
+
+extern "C" int psim_nccl_unique_id(void* out128) {
+  if (!out128) return PSIM_ERR_ARG;
+  if (!load_nccl()) return PSIM_ERR_NCCL;
+  ncclUniqueId id;
+  if (g_nccl.getUniqueId(&id) != ncclSuccess) return PSIM_ERR_NCCL;
+  memcpy(out128, &id, sizeof id);
   return PSIM_OK;
 }
 

@@ -113,14 +113,19 @@ __global__ void __launch_bounds__(256) update_kernel(UpdateArgs a) {
     const int64_t nsteps = e_b - ws;
     if (a.step >= nsteps) continue;
     const int64_t i = ws + a.step;
-    int f, c, s;
+    int f, c, s;          // latencies that drive the update
+    int pf = 0, pc = 0, ps = 0;   // the CNN's rounded prediction (recorded)
+    if (a.y) {
+      pf = lat_round(a.y[b * 3 + 0]);
+      pc = lat_round(a.y[b * 3 + 1]);
+      ps = lat_round(a.y[b * 3 + 2]);
+    }
     if (a.forced) {
       const uint16_t* p = a.forced + (i - a.row_lo) * 3;
       f = p[0]; c = p[1]; s = p[2];
+      if (!a.y) { pf = f; pc = c; ps = s; }
     } else {
-      f = lat_round(a.y[b * 3 + 0]);
-      c = lat_round(a.y[b * 3 + 1]);
-      s = lat_round(a.y[b * 3 + 2]);
+      f = pf; c = pc; s = ps;
     }
     int64_t clock = a.st.clock[b];
     const int k = a.st.count[b];
@@ -187,7 +192,7 @@ __global__ void __launch_bounds__(256) update_kernel(UpdateArgs a) {
       atomicAdd(a.st.k_hist + k, 1ull);
       if (i >= s_b) {
         const int64_t r = i - a.row_lo;
-        if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)f; a.rec_lat[3 * r + 1] = (uint16_t)c; a.rec_lat[3 * r + 2] = (uint16_t)s; }
+        if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
         if (a.rec_k) a.rec_k[r] = k;
         if (a.rec_clock) a.rec_clock[r] = clock;
       }
