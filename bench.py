@@ -43,6 +43,10 @@ CONFIGS = {
                desc="config2: 1M-instruction synthetic SPEC-like trace, 1024 sub-traces, W=1000, C3 CNN, bf16"),
     "c3": dict(L=100_000_000, N=65536, W=110, arch="C3", precision="bf16", seed_off=2,
                desc="config3: 100M-instruction synthetic SPEC-like trace, 65536 sub-traces, W=110, C3 CNN, bf16"),
+    # profiling stand-in: config 3's batch shape (65536 sub-traces, W=110) on a 4.2M-row
+    # prefix -> 174 lockstep steps with the same per-step kernel shapes (ncu runs only)
+    "c3p": dict(L=65536 * 64, N=65536, W=110, arch="C3", precision="bf16", seed_off=2,
+                desc="profiling: config3 batch shape on a 4.2M-row prefix (65536 sub-traces, W=110), C3, bf16"),
 }
 METRIC = "simulated instr/sec (MIPS, 8×B200 device-timed) + cycle error vs CPU oracle"
 REASONS = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
@@ -103,11 +107,17 @@ def roofline(stats, k_steps, cfg):
     avg_s = ms[dom] / 1e3 / max(launches[dom], 1)
     hist = np.array(stats["k_hist"], np.float64)
     kmean = float((hist * np.arange(112)).sum() / max(hist.sum(), 1))
+    fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0
     if names[dom].startswith("gemm_layer"):
         li = int(names[dom][-1])
         M, N, K = stats["layer_m"][li], stats["layer_n"][li], stats["layer_k"][li]
-        k_alg = 100 if li == 0 else K          # conv1: 2 rows x 50 real features (features padded to 64)
-        flops = 2.0 * M * N * k_alg
+        if fused and li == 0:     # conv_stack: per (sub-trace, position) block conv1 4x2x100x64 + conv2 2x2x128x128 + conv3 2x256x128
+            flops = float(M) * 247808.0
+        elif fused and li == 3:   # fc1 over P_tile positions (tile max of P_b), N = 256
+            flops = 2.0 * M * 256 * 128 * stats.get("mean_ptile", 5.0)
+        else:
+            k_alg = 100 if li == 0 else K      # conv1: 2 rows x 50 real features (features padded to 64)
+            flops = 2.0 * M * N * k_alg
         achieved = flops / avg_s / 1e12
         peak = pk["bf16_tflops_sustained"] if cfg["precision"] == "bf16" else 74.0
         out.update(bound="tensor", achieved=round(achieved, 2), peak=peak, unit="TFLOP/s",
@@ -124,6 +134,9 @@ def roofline(stats, k_steps, cfg):
                    frac=round(achieved / pk["hbm_gbs"], 4), bytes_per_launch=byts, peak_source=src + " hbm")
     out["traffic"] = ncu_traffic(names[dom])
     out["avg_launch_us"] = round(avg_s * 1e6, 2)
+    if fused:
+        out["kernel"] = {"gemm_layer0": "conv_stack_kernel (gather+conv1+conv2+conv3, fused)",
+                         "gemm_layer3": "fc1_head_kernel (fc1+head+update, fused)"}.get(names[dom], names[dom])
     out["kernels"] = {names[i]: {"ms": round(ms[i] / k_steps, 3), "launches": launches[i] // k_steps,
                                  "share": round(ms[i] / total_ms, 4) if total_ms else None}
                       for i in range(len(names)) if launches[i]}
@@ -185,6 +198,7 @@ def main():
     ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg (profiling runs)")
     args = ap.parse_args()
     cfg = CONFIGS[args.config]
     L, N, W = cfg["L"], cfg["N"], cfg["W"]
@@ -305,7 +319,7 @@ def main():
         line["roofline"] = roofline(stats, args.steps, cfg)
         line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces")}
         line["warmup_overhead"] = round(stats["simulated"] / stats["counted"] - 1, 4)
-    if rank == 0 and world == 1:
+    if rank == 0 and world == 1 and not args.no_cpu:
         # cpu_baseline: the oracle as it stands on a bounded sample of the same workload,
         # plus the sampled sub-traces' cycles vs the GPU (parity sample)
         n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W)

@@ -56,12 +56,15 @@ extern "C" {
                                 step and record the CNN's (f,c,s) in the per-row outputs, while the
                                 queue update follows the forced latencies (decision parity on a
                                 given trajectory, R17)                              */
+#define PSIM_LAYERWISE 8u    /* bf16 C3: use the layer-by-layer GEMM path instead of the fused
+                                padding-aware kernels (A/B comparison, parity of both)       */
 #define PSIM_PROFILE 2u      /* time every kernel class with CUDA events on the launch stream
                                 (psim_stats.kernel_ms / kernel_launches)                    */
 
 /* kernel classes reported in psim_stats.kernel_ms (names: psim_kernel_class_name) */
 #define PSIM_KC_GATHER 0
-#define PSIM_KC_LAYER0 1   /* first GEMM layer (conv1); layer i is PSIM_KC_LAYER0 + i */
+#define PSIM_KC_LAYER0 1   /* first GEMM layer (conv1); layer i is PSIM_KC_LAYER0 + i;
+                              fused path: 1 = conv_stack (gather+conv1-3), 4 = fc1_head (+update) */
 #define PSIM_KC_HEAD 5
 #define PSIM_KC_UPDATE 6
 #define PSIM_KC_OTHER 7

@@ -25,6 +25,7 @@ ARCH = {"M2": 1, "C3": 2, "RB7": 3}
 RECORD_ROWS = 1
 PROFILE = 2
 FORCE_PREDICT = 4
+LAYERWISE = 8
 MAX_CAP = 110
 NATTR = 47
 
@@ -162,7 +163,7 @@ class Simulator:
     def __init__(self, device: int = 0, precision: str = "bf16", queue_cap: int = MAX_CAP,
                  rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
                  stream=None, record_rows: bool = False, chunk_steps: int = 0, profile: bool = False,
-                 force_predict: bool = False):
+                 force_predict: bool = False, layerwise: bool = False):
         self._keep = []
         idbuf = None
         if nccl_id is not None:
@@ -174,7 +175,7 @@ class Simulator:
                   chunk_steps=chunk_steps,
                   stream=ctypes.c_void_p(int(stream)) if stream is not None else None,
                   flags=(RECORD_ROWS if record_rows else 0) | (PROFILE if profile else 0)
-                  | (FORCE_PREDICT if force_predict else 0))
+                  | (FORCE_PREDICT if force_predict else 0) | (LAYERWISE if layerwise else 0))
         h = ctypes.c_void_p()
         rc = lib().psim_create(ctypes.byref(o), ctypes.byref(h))
         if rc != OK:

@@ -1,0 +1,833 @@
+// fused_c3.cu -- the padding-aware fused step of the C3 ("3C+2F") model on
+// tcgen05 tensor cores (sm_100a).  Two kernels per lockstep step:
+//
+//  conv_stack_kernel   gather + conv1 + conv2 + conv3 for every VALID block
+//                      (sub-trace b, conv3 position p < P_b), never materialising
+//                      the 112x64 input in HBM; output a4[b][p][128] bf16.
+//  fc1_head_kernel     fc1 over the P_tile computed positions (+ the constant
+//                      table T[P_b] for the all-padding positions), ReLU, fc2,
+//                      rounding and the warp-level queue update; emits the
+//                      block list of the next step.
+//
+// Padding awareness generalises the paper's custom first convolution, which
+// "dynamically adjusts the dimensions of the convolution channel to perform
+// computation only over the non-paddings": with k = s = 2
+// convolutions a conv3 position p sees input rows 8p..8p+7 only, so every
+// position with 8p > k (all padding: PAPER.md:267, > 68% of rows) has the
+// same conv3 output c3 = conv3(conv2(conv1(0))), and its fc1 contribution is
+// folded into T[P] = b_fc1 + sum_{p >= P} Wfc1[:, p] c3 (R18).
+// P_b = ceil((k_b + 1) / 8).  Exact in real arithmetic; the oracle stays dense.
+//
+// conv_stack_kernel roles (416 threads): warps 0..3 = TMEM epilogues (bias,
+// ReLU, bf16) feeding the next layer's A operand in SWIZZLE_128B smem and the
+// coalesced a4 write-back; warp 4 = TMEM allocator + single-thread tcgen05.mma
+// issuer; warps 5..12 = gather (one thread per (block, row of the current conv1
+// position), all loads of a tile issued up front).  Weights W1/W2/W3
+// stay resident in smem (112 KB).  Per 128-block tile the MMA order is
+//   c1(0) c1(1) c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1) c3(1)
+// with K-split accumulation so A2 (16 KB) and A3 (32 KB) are single buffers.
+#include "internal.h"
+#include "sim_common.cuh"
+#include "tc_common.cuh"
+
+namespace psim {
+
+using namespace tc;
+
+// ------------------------------------------------------------ smem layout
+namespace cs {
+constexpr int TILE = 128;
+constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
+constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
+constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 4 atoms [128][64]
+constexpr int X_OFF = W3_OFF + 64 * 1024;    // 2 slots x 2 atoms [128][64]
+constexpr int A2_OFF = X_OFF + 64 * 1024;    // 1 atom  [128][64]
+constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
+constexpr int BAR_OFF = A3_OFF + 32 * 1024;  // mbarriers
+constexpr int BIAS_OFF = BAR_OFF + 256;      // b1[64] b2[128] b3[128] fp32
+constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
+constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 256, TMEM_COLS = 512;
+constexpr int THREADS = 448;   // warps 0-3 epilogue, 4 MMA, 5-12 gather, 13 a4 write-back
+constexpr int MMA_WARP = 4, GATHER_WARP0 = 5, WB_WARP = 13;
+}  // namespace cs
+
+struct ConvArgs {
+  const uint32_t* blocks;    // block ids (b << 4 | p) of this step
+  const uint32_t* nblocks;   // count of this step's list
+  uint32_t* next_count;      // the other step parity's counter, reset here
+  const uint8_t* trace;
+  int64_t row_lo, stride;
+  const int64_t* ws;
+  const int64_t* clock;
+  const int32_t* count;
+  const uint32_t* q_seq;
+  const uint32_t* q_fetch;
+  const uint32_t* q_cs;
+  int64_t step;
+  uint64_t qn;               // sub-traces (entry stride of the entry-major queue)
+  const __nv_bfloat16* w1;   // [64][128]
+  const __nv_bfloat16* w2;   // [128][128]
+  const __nv_bfloat16* w3;   // [128][256]
+  const float* b1;
+  const float* b2;
+  const float* b3;
+  __nv_bfloat16* a4;         // [n][14][128]
+  long long* dbg;            // optional stage timestamps of CTA 0 (PSIM_DEBUG_TIMING), else nullptr
+};
+
+// debug timestamps: dbg[tile * 256 + slot] = clock64() for CTA 0, first 4 tiles
+#define PSIM_TS(slot)                                                                                   \
+  do {                                                                                                 \
+    if (a.dbg && blockIdx.x == 0 && it < 4 && lane == 0) a.dbg[it * 256 + (slot)] = clock64();        \
+  } while (0)
+
+__device__ __forceinline__ uint32_t bf16_bits_u8(uint32_t v) {   // exact: v < 256
+  return __float_as_uint((float)v) >> 16;
+}
+__device__ __forceinline__ uint32_t bf16_bits_int(int v) {       // RNE (time features up to 8190)
+  return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn((float)v));
+}
+
+// load a [rows][K] bf16 row-major weight into K-major SW128 atoms ([rows][64] each)
+__device__ void load_weight_sw128(uint8_t* dst, const __nv_bfloat16* w, int rows, int K, int tid, int nthr) {
+  const int chunks_per_row = K / 8;   // 16-byte chunks
+  const int total = rows * chunks_per_row;
+  const uint4* src = reinterpret_cast<const uint4*>(w);
+  for (int idx = tid; idx < total; idx += nthr) {
+    const int r = idx / chunks_per_row, ch = idx % chunks_per_row;
+    const int atom = ch / 8, c = ch % 8;
+    st_sw128(dst + atom * rows * 128, r, c, __ldg(src + idx));
+  }
+}
+
+__global__ void __launch_bounds__(cs::THREADS, 1)
+    conv_stack_kernel(ConvArgs a, const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2,
+                      const __grid_constant__ CUtensorMap tmW3) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
+  uint64_t* xfull = bars + 0;    // [2]  8 gather warps
+  uint64_t* xempty = bars + 2;   // [2]  commit
+  uint64_t* c1full = bars + 4;   // [2]  commit
+  uint64_t* c1empty = bars + 6;  // [2]  4 epilogue warps
+  uint64_t* a2full = bars + 8;   //      4
+  uint64_t* a2empty = bars + 9;  //      commit
+  uint64_t* c2full = bars + 10;  //      commit
+  uint64_t* c2empty = bars + 11; //      4
+  uint64_t* a3full = bars + 12;  //      4
+  uint64_t* a3empty = bars + 13; //      commit
+  uint64_t* c3full = bars + 14;  //      commit
+  uint64_t* c3empty = bars + 15; //      4
+  uint64_t* wbar = bars + 16;    //      weights landed (TMA)
+  uint64_t* stg_full = bars + 17;   //   4: conv3 rows staged in the A3 region
+  uint64_t* stg_empty = bars + 18;  //   1: write-back warp done reading the staging rows
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 19);
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint32_t nblocks = *a.nblocks;
+  const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
+  if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
+
+  if (tid == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(xfull + i, 8); mbar_init(xempty + i, 1);
+      mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
+    }
+    mbar_init(a2full, 4); mbar_init(a2empty, 1); mbar_init(c2full, 1); mbar_init(c2empty, 4);
+    mbar_init(a3full, 4); mbar_init(a3empty, 1); mbar_init(c3full, 1); mbar_init(c3empty, 4);
+    mbar_init(wbar, 1);
+    mbar_init(stg_full, 4); mbar_init(stg_empty, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    // resident weights W1/W2/W3 (112 KB) by TMA, already in the SWIZZLE_128B operand layout
+    mbar_expect_tx(wbar, 112 * 1024 + 1280);
+    float* sbias = reinterpret_cast<float*>(sm + cs::BIAS_OFF);
+    bulk_g2s(sbias, a.b1, 256, wbar);
+    bulk_g2s(sbias + 64, a.b2, 512, wbar);
+    bulk_g2s(sbias + 192, a.b3, 512, wbar);
+    for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W1_OFF + kc * 8192, &tmW1, wbar, kc * 64, 0);
+    for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W2_OFF + kc * 16384, &tmW2, wbar, kc * 64, 0);
+    for (int kc = 0; kc < 4; ++kc) tma_load_2d(sm + cs::W3_OFF + kc * 16384, &tmW3, wbar, kc * 64, 0);
+  }
+  if (warp == cs::MMA_WARP) tmem_alloc(tmem_slot, cs::TMEM_COLS);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+  mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
+  const float* sb1 = reinterpret_cast<const float*>(sm + cs::BIAS_OFF);
+  const float* sb2 = sb1 + 64;
+  const float* sb3 = sb1 + 192;
+
+  if (warp == cs::MMA_WARP) {
+    if (lane == 0) {   // ============================ MMA issuer
+      const uint32_t sbase = smem_u32(sm);
+      const uint32_t id64 = idesc_bf16(128, 64), id128 = idesc_bf16(128, 128);
+      uint32_t it = 0;
+      for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+        auto c1 = [&](int j) {
+          const int s = j & 1;
+          const uint32_t n = it * 2 + (j >> 1);
+          PSIM_TS(0 + 2 * j);
+          wait_full(xfull + s, n);
+          wait_empty(c1empty + s, n);
+          PSIM_TS(1 + 2 * j);
+          fence_after();
+          const uint32_t xa = sbase + cs::X_OFF + s * 32768;
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
+                     sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
+          mma_commit(xempty + s);
+          mma_commit(c1full + s);
+        };
+        auto c2 = [&](int h, int kh) {
+          const uint32_t n = it * 4 + h * 2 + kh;
+          PSIM_TS(8 + 2 * (h * 2 + kh));
+          wait_full(a2full, n);
+          if (kh == 0) wait_empty(c2empty, it * 2 + h);
+          PSIM_TS(9 + 2 * (h * 2 + kh));
+          fence_after();
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            mma_bf16(tmem + cs::TMEM_C2, sw128_desc(sbase + cs::A2_OFF + k * 32),
+                     sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
+          mma_commit(a2empty);
+          if (kh == 1) mma_commit(c2full);
+        };
+        auto c3 = [&](int kh) {
+          PSIM_TS(16 + 2 * kh);
+          wait_full(a3full, it * 2 + kh);
+          if (kh == 0) wait_empty(c3empty, it);
+          PSIM_TS(17 + 2 * kh);
+          fence_after();
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            mma_bf16(tmem + cs::TMEM_C3, sw128_desc(sbase + cs::A3_OFF + (k >> 2) * 16384 + (k & 3) * 32),
+                     sw128_desc(sbase + cs::W3_OFF + (2 * kh + (k >> 2)) * 16384 + (k & 3) * 32), id128,
+                     (kh | k) != 0);
+          mma_commit(a3empty);
+          if (kh == 1) mma_commit(c3full);
+        };
+        c1(0); c1(1); c2(0, 0); c2(0, 1); c1(2); c1(3); c3(0); c2(1, 0); c2(1, 1); c3(1);
+        PSIM_TS(20);
+      }
+    }
+  } else if (warp < 4) {   // ============================ epilogues
+    const int q = warp & 3;
+    const int m = q * 32 + lane;                    // tile row = TMEM lane
+    const uint32_t lane_base = (uint32_t)(q * 32) << 16;
+    uint32_t it = 0;
+    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+      auto e1 = [&](int j) {   // C1 (64 fp32) -> relu(+b1) -> bf16 -> A2
+        const int s = j & 1;
+        if (q == 0) PSIM_TS(32 + 4 * j);
+        wait_full(c1full + s, it * 2 + (j >> 1));
+        if (q == 0) PSIM_TS(33 + 4 * j);
+        fence_after();
+        uint32_t pk[32];
+        {
+          uint32_t r0[32], r1[32];
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C1 + s * 64, r0);
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C1 + s * 64 + 32, r1);
+          tmem_wait_ld();
+#pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb1[2 * c], 0.f),
+                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb1[2 * c + 1], 0.f));
+            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb1[32 + 2 * c], 0.f),
+                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb1[33 + 2 * c], 0.f));
+          }
+        }
+        fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(c1empty + s);
+        if (q == 0) PSIM_TS(34 + 4 * j);
+        wait_empty(a2empty, it * 4 + j);
+        if (q == 0) PSIM_TS(35 + 4 * j);
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+          st_sw128(sm + cs::A2_OFF, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(a2full);
+        if (q == 0) PSIM_TS(48 + j);
+      };
+      auto e2 = [&](int h) {   // C2 (128 fp32) -> relu(+b2) -> bf16 -> A3 (2 atoms)
+        if (q == 0) PSIM_TS(56 + 4 * h);
+        wait_full(c2full, it * 2 + h);
+        if (q == 0) PSIM_TS(57 + 4 * h);
+        fence_after();
+        wait_empty(a3empty, it * 2 + h);
+        if (h == 0) wait_empty(stg_empty, it);        // previous tile's staging rows written back
+        if (q == 0) PSIM_TS(58 + 4 * h);
+#pragma unroll 1
+        for (int cp = 0; cp < 2; ++cp) {              // 2 x (two TMEM loads in flight, one wait)
+          uint32_t r0[32], r1[32];
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + cp * 64, r0);
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + cp * 64 + 32, r1);
+          tmem_wait_ld();
+          uint32_t pk[32];
+#pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb2[cp * 64 + 2 * c], 0.f),
+                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb2[cp * 64 + 2 * c + 1], 0.f));
+            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb2[cp * 64 + 32 + 2 * c], 0.f),
+                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb2[cp * 64 + 33 + 2 * c], 0.f));
+          }
+          uint8_t* atom = sm + cs::A3_OFF + cp * 16384;   // 64 channels per atom
+#pragma unroll
+          for (int c = 0; c < 8; ++c)
+            st_sw128(atom, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
+        }
+        fence_before();
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) { mbar_arrive(c2empty); mbar_arrive(a3full); }
+        if (q == 0) PSIM_TS(59 + 4 * h);
+      };
+      auto e3 = [&]() {        // C3 (128 fp32) -> relu(+b3) -> bf16 -> A3 staging rows -> write-back warp
+        if (q == 0) PSIM_TS(64);
+        wait_full(c3full, it);   // c3 done: A3 is free for staging
+        if (q == 0) PSIM_TS(65);
+        fence_after();
+        uint8_t* row = sm + cs::A3_OFF + m * 256;     // plain row-major staging [128][256 B]
+#pragma unroll 1
+        for (int cp = 0; cp < 2; ++cp) {
+          uint32_t r0[32], r1[32];
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64, r0);
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64 + 32, r1);
+          tmem_wait_ld();
+          uint32_t pk[32];
+#pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb3[cp * 64 + 2 * c], 0.f),
+                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb3[cp * 64 + 2 * c + 1], 0.f));
+            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb3[cp * 64 + 32 + 2 * c], 0.f),
+                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb3[cp * 64 + 33 + 2 * c], 0.f));
+          }
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {   // lane-rotated chunk order: conflict-free 256-B row pitch
+            const int sel = (c + m) & 7;
+            uint4 v = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+#pragma unroll
+            for (int t = 1; t < 8; ++t)
+              if (sel == t) v = make_uint4(pk[4 * t], pk[4 * t + 1], pk[4 * t + 2], pk[4 * t + 3]);
+            *reinterpret_cast<uint4*>(row + (cp * 8 + sel) * 16) = v;
+          }
+          if (q == 0) PSIM_TS(67 + cp);
+        }
+        fence_before();
+        fence_async_smem();                           // staging rows are read by TMA bulk copies
+        __syncwarp();
+        if (lane == 0) { mbar_arrive(c3empty); mbar_arrive(stg_full); }
+        if (q == 0) PSIM_TS(66);
+      };
+      // same order as the MMA issue schedule: e1(0) e1(1) e2(0) e1(2) e1(3) e2(1) e3
+#pragma unroll 1
+      for (int ev = 0; ev < 7; ++ev) {
+        if (ev == 2 || ev == 5) e2(ev == 5);
+        else if (ev == 6) e3();
+        else e1(ev < 2 ? ev : ev - 1);
+      }
+    }
+  } else if (warp == cs::WB_WARP) {   // ============================ a4 write-back
+    // copies the 128 staged conv3 rows (256 B each) of a tile to a4[b][p] with
+    // coalesced 256-B stores, off the epilogue's critical path
+    uint32_t it = 0;
+    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+      uint32_t ids[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t bi = tl * cs::TILE + u * 32 + lane;
+        ids[u] = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
+      }
+      wait_full(stg_full, it);
+#pragma unroll
+      for (int u = 0; u < 4; ++u)                   // one 256-B TMA bulk store per row
+        if (ids[u] != 0xFFFFFFFFu)
+          bulk_s2g(a.a4 + ((uint64_t)(ids[u] >> 4) * 14 + (ids[u] & 15)) * 128,
+                   sm + cs::A3_OFF + (u * 32 + lane) * 256, 256);
+      bulk_commit();
+      bulk_wait_read();                             // staging rows consumed -> A3 reusable
+      __syncwarp();
+      if (lane == 0) mbar_arrive(stg_empty);
+    }
+  } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
+    // Thread (m, h) builds row 2j+h of block m for the 4 conv1 positions j of a
+    // tile.  All loads of a tile are issued up front (block id -> sub-trace state
+    // -> 4 queue entries -> 4 trace rows: 3 dependent round trips per tile
+    // instead of 8), then rows are converted into the A tile as X slots free up.
+    const int g = tid - cs::GATHER_WARP0 * 32;
+    const int m = g & 127, h = g >> 7;
+    uint32_t it = 0;
+    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+      const uint32_t bi = tl * cs::TILE + m;
+      const bool valid = bi < nblocks;
+      uint32_t b = 0, p = 0;
+      int k = -1;
+      int64_t i = 0;
+      uint32_t clo = 0;
+      if (valid) {
+        const uint32_t id = a.blocks[bi];
+        b = id >> 4; p = id & 15;
+        k = a.count[b];
+        i = a.ws[b] + a.step;
+        clo = (uint32_t)a.clock[b];
+      }
+      if (warp == cs::GATHER_WARP0) PSIM_TS(80);
+      int64_t rowj[4];
+      int tf[4][3];
+      bool on[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int R = (int)p * 8 + 2 * j + h;        // input row of this thread
+        on[j] = valid && R <= k;
+        rowj[j] = i;                                 // R == 0: current instruction first
+        tf[j][0] = tf[j][1] = tf[j][2] = 0;
+        if (on[j] && R > 0) {
+          const int e = k - R;                       // context newest first (R6)
+          const uint64_t qo = (uint64_t)e * a.qn + b;
+          rowj[j] = a.q_seq[qo];
+          const uint32_t csv = a.q_cs[qo];
+          const int c = csv & 0xFFFF, sv = csv >> 16;
+          int age = (int)(clo - a.q_fetch[qo]);      // time relative to Clock (R2)
+          int remc = max(0, c - age);
+          int remr = c + sv - age;
+          tf[j][0] = min(age, kTimeMax); tf[j][1] = min(remc, kTimeMax); tf[j][2] = min(remr, kTimeMax);
+        }
+      }
+      uint4 v[4][3];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (on[j]) {
+          const uint4* ar = reinterpret_cast<const uint4*>(a.trace + (rowj[j] - a.row_lo) * a.stride);
+          v[j][0] = __ldg(ar); v[j][1] = __ldg(ar + 1); v[j][2] = __ldg(ar + 2);
+        } else {
+          v[j][0] = v[j][1] = v[j][2] = make_uint4(0, 0, 0, 0);
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int s = j & 1;
+        uint32_t w[32];                              // 64 bf16 values, packed pairs
+#pragma unroll
+        for (int t = 0; t < 32; ++t) w[t] = 0;
+        if (on[j]) {
+          uint32_t by[12];
+          by[0] = v[j][0].x; by[1] = v[j][0].y; by[2] = v[j][0].z; by[3] = v[j][0].w;
+          by[4] = v[j][1].x; by[5] = v[j][1].y; by[6] = v[j][1].z; by[7] = v[j][1].w;
+          by[8] = v[j][2].x; by[9] = v[j][2].y; by[10] = v[j][2].z; by[11] = v[j][2].w;
+#define PSIM_BYTE(idx) ((by[(idx) >> 2] >> (((idx) & 3) * 8)) & 0xFFu)
+          // columns: 0..2 time, 3..49 attributes 0..46, 50..63 zero (R1)
+          w[0] = bf16_bits_int(tf[j][0]) | (bf16_bits_int(tf[j][1]) << 16);
+          w[1] = bf16_bits_int(tf[j][2]) | (bf16_bits_u8(PSIM_BYTE(0)) << 16);
+#pragma unroll
+          for (int t = 2; t < 25; ++t)   // columns 2t, 2t+1 -> attributes 2t-3, 2t-2
+            w[t] = bf16_bits_u8(PSIM_BYTE(2 * t - 3)) | (bf16_bits_u8(PSIM_BYTE(2 * t - 2)) << 16);
+#undef PSIM_BYTE
+        }
+        if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+        wait_empty(xempty + s, it * 2 + (j >> 1));
+        if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
+        uint8_t* atom = sm + cs::X_OFF + s * 32768 + h * 16384;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) st_sw128(atom, m, c, make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]));
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(xfull + s);
+        if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == cs::MMA_WARP) {
+    fence_after();
+    tmem_dealloc(tmem, cs::TMEM_COLS);
+  }
+}
+
+// ============================================================ fc1 / head / update
+namespace fh {
+constexpr int BM = 128, BN = 256, BK = 64;
+constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
+constexpr int STAGES = 4;
+constexpr int T_STRIDE = 260;                 // padded rows of the constant table (bank spread, 16-B rows)
+constexpr int T_OFF = STAGES * STAGE;         // float [15][257]
+constexpr int W2_OFF = T_OFF + 15 * T_STRIDE * 4;   // float [3][256] + bias[3]
+constexpr int Y_OFF = W2_OFF + (3 * 256 + 4) * 4;   // float [128][3]
+constexpr int P_OFF = Y_OFF + 2 * 128 * 3 * 4;      // int [2][16] tile scan scratch per update group
+constexpr int H_OFF = P_OFF + 32 * 4;               // uint [112] k histogram of this CTA
+constexpr int BAR_OFF = (H_OFF + 112 * 4 + 7) & ~7;
+constexpr int SMEM = BAR_OFF + 160 + 1024;
+constexpr int THREADS = 448;   // warp 0 TMA, 1 MMA, 2-5 epilogue (F -> y), 6-9 / 10-13 update groups (even / odd tiles)
+}  // namespace fh
+
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+struct HeadArgs {
+  UpdateArgs u;              // state, step, cap, forced, records (y unused)
+  const int64_t* e;
+  const uint8_t* tileP;      // [ntiles] P_tile of this step
+  uint8_t* tileP_next;       // [ntiles] P_tile of the next step
+  uint32_t* blocks_next;     // block list of the next step
+  uint32_t* next_count;
+  __nv_bfloat16* a4;         // [n][14][128] (zero-fill of [P_b, P_tile) for the next step)
+  const float* T;            // [15][256] constant table
+  const float* w2;           // [3][256]
+  const float* b2;           // [3]
+  int force_predict;         // run the head even when teacher-forced
+  long long* dbg;            // optional timestamps (PSIM_DEBUG_TIMING), slots 128..
+};
+
+__global__ void __launch_bounds__(fh::THREADS, 1)
+    fc1_head_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, HeadArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  float* sT = reinterpret_cast<float*>(sm + fh::T_OFF);
+  float* sW2 = reinterpret_cast<float*>(sm + fh::W2_OFF);
+  int* sP = reinterpret_cast<int*>(sm + fh::P_OFF);
+  unsigned int* sHist = reinterpret_cast<unsigned int*>(sm + fh::H_OFF);
+  uint64_t* full = reinterpret_cast<uint64_t*>(sm + fh::BAR_OFF);
+  uint64_t* empty = full + fh::STAGES;
+  uint64_t* tfull = empty + fh::STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = nullptr;
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint64_t n = a.u.st.n;
+  const uint32_t ntiles = (uint32_t)((n + fh::BM - 1) / fh::BM);
+
+  uint64_t* cbar = tempty + 2;   // constant table + fc2 landed (bulk copies)
+  uint64_t* yfull = cbar + 1;    // [2] epilogue -> update: y of a tile in sY[buf]
+  uint64_t* yempty = yfull + 2;  // [2] update -> epilogue: sY[buf] consumed
+  float* sY = reinterpret_cast<float*>(sm + fh::Y_OFF);
+  tmem_slot = reinterpret_cast<uint32_t*>(yempty + 2);
+  if (tid < 3) sW2[768 + tid] = a.b2[tid];
+  for (int idx = tid; idx < 112; idx += fh::THREADS) sHist[idx] = 0;
+  if (tid == 0) {
+    for (int s = 0; s < fh::STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(tfull + i, 1); mbar_init(tempty + i, 4); }
+    mbar_init(cbar, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(yfull + i, 4); mbar_init(yempty + i, 4); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    mbar_expect_tx(cbar, 15 * 1024 + 3 * 1024);
+    for (int r = 0; r < 15; ++r) bulk_g2s(sT + r * fh::T_STRIDE, a.T + r * 256, 1024, cbar);
+    bulk_g2s(sW2, a.w2, 3 * 1024, cbar);
+  }
+  if (warp == 1) tmem_alloc(tmem_slot, 512);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const bool run_head = (a.u.forced == nullptr) || a.force_predict;
+  if (warp >= 2 && warp < 6) mbar_wait(cbar, 0);   // epilogue warps read T and fc2 from smem
+
+  if (warp == 0) {
+    if (lane == 0 && run_head) {   // ---- TMA producer
+      uint32_t stage = 0, phase = 0;
+      uint32_t it = 0;
+      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
+        const int nk = 2 * a.tileP[tt];
+        PSIM_TS(128);
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(empty + stage, phase ^ 1);
+          uint8_t* sa = sm + stage * fh::STAGE;
+          mbar_expect_tx(full + stage, fh::STAGE);
+          tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
+          tma_load_2d(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0);
+          if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
+        }
+        PSIM_TS(129);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && run_head) {   // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_bf16(fh::BM, fh::BN);
+      uint32_t stage = 0, phase = 0, it = 0;
+      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
+        const int nk = 2 * a.tileP[tt];
+        const int acc = it & 1;
+        PSIM_TS(132);
+        wait_empty(tempty + acc, it >> 1);
+        PSIM_TS(133);
+        fence_after();
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(full + stage, phase);
+          fence_after();
+          const uint32_t sa = smem_u32(sm + stage * fh::STAGE), sb = sa + fh::A_BYTES;
+#pragma unroll
+          for (int k = 0; k < fh::BK / 16; ++k)
+            mma_bf16(tmem + acc * fh::BN, sw128_desc(sa + 32 * k), sw128_desc(sb + 32 * k), idesc, (kb | k) != 0);
+          mma_commit(empty + stage);
+          if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
+        }
+        mma_commit(tfull + acc);   // nk == 0: arrives once the earlier MMAs are done
+        PSIM_TS(134);
+      }
+    }
+  } else if (warp < 6) {   // ---- epilogue (warps 2..5): F -> relu(F + T[P_b]) . fc2 -> y in smem
+    const int q = warp & 3;
+    const int m = q * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(q * 32) << 16;
+    uint32_t it = 0;
+    for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
+      const int acc = it & 1, yb = it & 1;
+      const uint64_t b = (uint64_t)tt * fh::BM + m;
+      const int ptile = a.tileP[tt];
+      const int kb = b < n ? a.u.st.count[b] : 0;   // read before this tile's update (y handoff orders it)
+      const int pb = min((kb + 8) >> 3, 14);        // computed positions of this sub-trace
+      float y0 = 0.f, y1 = 0.f, y2 = 0.f;
+      if (q == 2) PSIM_TS(140);
+      if (run_head) {
+        wait_full(tfull + acc, it >> 1);
+        if (q == 2) PSIM_TS(141);
+        fence_after();
+        y0 = sW2[768]; y1 = sW2[769]; y2 = sW2[770];
+        const float* Trow = sT + pb * fh::T_STRIDE;
+        // fc1 = F (positions < P_tile; rows [P_b, P_tile) are zero) + T[P_b]; ReLU; fc2 (R16, R18)
+#pragma unroll 1
+        for (int cc = 0; cc < fh::BN / 32; ++cc) {
+          uint32_t r0[32];
+          tmem_ld32(tmem + lane_base + acc * fh::BN + cc * 32, r0);
+#pragma unroll
+          for (int j4 = 0; j4 < 8; ++j4) {
+            const int col = cc * 32 + j4 * 4;
+            const float4 tv = *reinterpret_cast<const float4*>(Trow + col);
+            const float4 w0 = *reinterpret_cast<const float4*>(sW2 + col);
+            const float4 w1 = *reinterpret_cast<const float4*>(sW2 + 256 + col);
+            const float4 w2v = *reinterpret_cast<const float4*>(sW2 + 512 + col);
+            const float f0 = ptile > 0 ? __uint_as_float(r0[j4 * 4]) : 0.f, f1 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 1]) : 0.f;
+            const float f2 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 2]) : 0.f, f3 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 3]) : 0.f;
+            const float h0 = fmaxf(f0 + tv.x, 0.f), h1 = fmaxf(f1 + tv.y, 0.f);
+            const float h2 = fmaxf(f2 + tv.z, 0.f), h3 = fmaxf(f3 + tv.w, 0.f);
+            y0 = fmaf(h0, w0.x, y0); y0 = fmaf(h1, w0.y, y0); y0 = fmaf(h2, w0.z, y0); y0 = fmaf(h3, w0.w, y0);
+            y1 = fmaf(h0, w1.x, y1); y1 = fmaf(h1, w1.y, y1); y1 = fmaf(h2, w1.z, y1); y1 = fmaf(h3, w1.w, y1);
+            y2 = fmaf(h0, w2v.x, y2); y2 = fmaf(h1, w2v.y, y2); y2 = fmaf(h2, w2v.z, y2); y2 = fmaf(h3, w2v.w, y2);
+          }
+        }
+        fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tempty + acc);
+      }
+      wait_empty(yempty + yb, it >> 1);
+      float* yrow = sY + (yb * 128 + m) * 3;
+      yrow[0] = y0; yrow[1] = y1; yrow[2] = y2;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(yfull + yb);
+      if (q == 2) PSIM_TS(142);
+    }
+  } else {   // ---- update (group 0: warps 6..9 even tiles, group 1: 10..13 odd tiles), thread per sub-trace
+    const int grp = (warp - 6) >> 2;
+    const int q = (warp - 6) & 3;
+    const int m = q * 32 + lane;
+    int* sPg = sP + grp * 16;
+    uint32_t it = grp;
+    for (uint32_t tt = blockIdx.x + grp * gridDim.x; tt < ntiles; tt += 2 * gridDim.x, it += 2) {
+      const int yb = it & 1;
+      const uint64_t b = (uint64_t)tt * fh::BM + m;
+      const bool inb = b < n;
+      int64_t ws = 0, s_b = 0, nsteps = 0, clock = 0;
+      int kb = 0;
+      if (inb) {   // prefetch the state and the first queue entries while the head runs
+        ws = a.u.st.ws[b]; s_b = a.u.st.s[b]; nsteps = a.e[b] - ws;
+        kb = a.u.st.count[b]; clock = a.u.st.clock[b];
+      }
+      const bool active = inb && a.u.step < nsteps;
+      QBatch first;
+      if (active) load_qbatch(a.u.st, b, kb, first);
+      const int pb = min((kb + 8) >> 3, 14);
+      wait_full(yfull + yb, it >> 1);
+      const float* yrow = sY + (yb * 128 + m) * 3;
+      const float y0 = yrow[0], y1 = yrow[1], y2 = yrow[2];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(yempty + yb);
+      int pnext = 0;
+      if (active) {
+        const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, first, run_head, y0, y1, y2, sHist);
+        if (a.u.step + 1 < nsteps) {
+          pnext = (knew + 8) >> 3;                 // ceil((k+1)/8)
+          // keep a4 rows >= P_b zero: clear the rows this sub-trace no longer computes
+          for (int p = pnext; p < pb; ++p) {
+            uint4* dst = reinterpret_cast<uint4*>(a.a4 + (b * 14 + p) * 128);
+#pragma unroll
+            for (int c = 0; c < 16; ++c) dst[c] = make_uint4(0, 0, 0, 0);
+          }
+        }
+      }
+      if (q == 0 && grp == 0) PSIM_TS(143);
+      // tile-wide scan of pnext: one atomic per tile reserves the block-list range
+      int incl = pnext;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+      }
+      int wmax = pnext;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) wmax = max(wmax, __shfl_xor_sync(0xffffffffu, wmax, o));
+      if (lane == 31) { sPg[q] = incl; sPg[4 + q] = wmax; }
+      named_bar_sync(2 + grp, 128);
+      int before = 0;
+      for (int w2 = 0; w2 < q; ++w2) before += sPg[w2];
+      if (m == 0) {
+        const int total = sPg[0] + sPg[1] + sPg[2] + sPg[3];
+        sPg[8] = total ? (int)atomicAdd(a.next_count, (uint32_t)total) : 0;
+        a.tileP_next[tt] = (uint8_t)max(max(sPg[4], sPg[5]), max(sPg[6], sPg[7]));
+      }
+      named_bar_sync(2 + grp, 128);
+      const uint32_t base = (uint32_t)sPg[8] + (uint32_t)(before + incl - pnext);
+      if (q == 0 && grp == 0) PSIM_TS(144);
+      for (int p = 0; p < pnext; ++p) a.blocks_next[base + p] = (uint32_t)(b << 4) | (uint32_t)p;
+      named_bar_sync(2 + grp, 128);   // sP reused by the next tile
+    }
+  }
+  __syncthreads();
+  for (int k = tid; k < 112; k += fh::THREADS)
+    if (sHist[k]) atomicAdd(a.u.st.k_hist + k, (unsigned long long)sHist[k]);
+  fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    fence_after();
+    tmem_dealloc(tmem, 512);
+  }
+}
+
+// step-0 block list: every sub-trace has k = 0 -> P = 1
+__global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count, uint8_t* tileP, uint32_t* next_count) {
+  const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (t < n) blocks[t] = (uint32_t)(t << 4);
+  if (t < (n + 127) / 128) tileP[t] = 1;
+  if (t == 0) { *count = (uint32_t)n; *next_count = 0; }
+}
+
+// ---------------------------------------------------------------- host side
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_fn2() {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+static bool map2d(CUtensorMap* m, const void* ptr, uint64_t rows, uint64_t cols, uint32_t box_rows) {
+  EncodeTiledFn fn = encode_fn2();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {cols * 2};
+  cuuint32_t box[2] = {64, box_rows};
+  cuuint32_t es[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static int sm_count() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st) {
+  const uint64_t th = n > 1 ? n : 1;
+  fused_init_kernel<<<(unsigned)((th + 255) / 256), 256, 0, st>>>(n, f.blocks, f.count + 0, f.tileP[0], f.count + 1);
+}
+
+// PSIM_DEBUG_TIMING=<step>: CTA 0 of conv_stack records clock64() at every
+// pipeline event of its first 4 tiles of that step (dumped to
+// $PSIM_DEBUG_TIMING_OUT by fused_dump_debug).  Off by default.
+static long long* g_dbg = nullptr;
+static int64_t g_dbg_step = -2;
+static long long* debug_buffer(int64_t step) {
+  if (g_dbg_step == -2) {
+    const char* e = getenv("PSIM_DEBUG_TIMING");
+    g_dbg_step = e ? atoll(e) : -1;
+    if (g_dbg_step >= 0) { cudaMalloc(&g_dbg, 4 * 256 * 8); cudaMemset(g_dbg, 0, 4 * 256 * 8); }
+  }
+  return (g_dbg_step >= 0 && step == g_dbg_step) ? g_dbg : nullptr;
+}
+void fused_dump_debug() {
+  const char* out = getenv("PSIM_DEBUG_TIMING_OUT");
+  if (!g_dbg || !out) return;
+  long long h[4 * 256];
+  cudaMemcpy(h, g_dbg, sizeof h, cudaMemcpyDeviceToHost);
+  FILE* f = fopen(out, "w");
+  if (!f) return;
+  for (int t = 0; t < 4; ++t)
+    for (int sidx = 0; sidx < 256; ++sidx)
+      if (h[t * 256 + sidx]) fprintf(f, "%d %d %lld\n", t, sidx, h[t * 256 + sidx]);
+  fclose(f);
+}
+
+void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(conv_stack_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, cs::SMEM);
+    attr = true;
+  }
+  ConvArgs a;
+  a.blocks = f.blocks;
+  a.nblocks = f.count + (step & 1);
+  a.next_count = f.count + ((step + 1) & 1);
+  a.trace = g.trace; a.row_lo = g.row_lo; a.stride = g.stride;
+  a.ws = g.ws; a.clock = g.clock; a.count = g.count;
+  a.q_seq = g.q_seq; a.q_fetch = g.q_fetch; a.q_cs = g.q_cs;
+  a.step = step;
+  a.qn = g.n;
+  a.w1 = f.w1; a.w2 = f.w2; a.w3 = f.w3;
+  a.b1 = f.b1; a.b2 = f.b2; a.b3 = f.b3;
+  a.a4 = f.a4;
+  a.dbg = debug_buffer(step);
+  // the block count is only known on the device: launch one persistent CTA per SM
+  // (n*14 blocks at most); CTAs with no tile exit after setup.
+  const uint64_t max_tiles = (n * 14 + cs::TILE - 1) / cs::TILE;
+  const int grid = (int)std::min<uint64_t>(max_tiles, (uint64_t)sm_count());
+  conv_stack_kernel<<<grid, cs::THREADS, cs::SMEM, st>>>(a, f.mapW1, f.mapW2, f.mapW3);
+}
+
+void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
+                     cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(fc1_head_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, fh::SMEM);
+    attr = true;
+  }
+  HeadArgs a;
+  a.u = u;
+  a.e = e;
+  a.tileP = f.tileP[step & 1];
+  a.tileP_next = f.tileP[(step + 1) & 1];
+  a.blocks_next = f.blocks;   // conv_stack of this step has finished with the list
+  a.next_count = f.count + ((step + 1) & 1);
+  a.a4 = f.a4;
+  a.T = f.T; a.w2 = f.head_w; a.b2 = f.head_b;
+  a.force_predict = force_predict ? 1 : 0;
+  a.dbg = debug_buffer(step);
+  const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
+  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
+  fc1_head_kernel<<<grid, fh::THREADS, fh::SMEM, st>>>(f.mapA, f.mapB, a);
+}
+
+bool fused_make_weight_maps(FusedC3& f) {
+  return map2d(&f.mapW1, f.w1, 64, 128, 64) && map2d(&f.mapW2, f.w2, 128, 128, 128) &&
+         map2d(&f.mapW3, f.w3, 128, 256, 128);
+}
+
+bool fused_make_maps(FusedC3& f, uint64_t n) {
+  return map2d(&f.mapA, f.a4, n, 14 * 128, fh::BM) && map2d(&f.mapB, f.wfc1, 256, 14 * 128, fh::BN);
+}
+
+}  // namespace psim

@@ -3,6 +3,7 @@
 // nothing here is shared with oracle/.
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
@@ -54,9 +55,11 @@ struct SimState {
   int64_t* bnd = nullptr;       // [n] Clock at the end of warm-up
   int64_t* cycles = nullptr;    // [n] Clock_end - bnd
   int32_t* count = nullptr;     // [n] live context entries
-  uint32_t* q_seq = nullptr;    // [n][kQStride] global row index of each live entry (fetch order)
-  uint32_t* q_fetch = nullptr;  // [n][kQStride] low 32 bits of the fetch Clock
-  uint32_t* q_cs = nullptr;     // [n][kQStride] c | s << 16
+  // queue entries are ENTRY-MAJOR: entry e of sub-trace b at [e * n + b], so the
+  // threads of a warp (consecutive sub-traces) touch consecutive words
+  uint32_t* q_seq = nullptr;    // [kQStride][n] global row index of each live entry (fetch order)
+  uint32_t* q_fetch = nullptr;  // [kQStride][n] low 32 bits of the fetch Clock
+  uint32_t* q_cs = nullptr;     // [kQStride][n] c | s << 16
   unsigned long long* k_hist = nullptr;   // [112]
   unsigned long long* stalls = nullptr;   // [1]
   long long* total = nullptr;             // [1] local sum of cycles (NCCL send/recv buffer)
@@ -121,6 +124,34 @@ void launch_gemm_tc(const __nv_bfloat16* A, const void* Wtc, const float* b, voi
                     bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st);
 // Pre-tile a [N][K] bf16 weight for the tensor-core kernel (device -> device).
 void* pretile_weight_tc(const __nv_bfloat16* W, int N, int K, cudaStream_t st);
+
+// ---- fused padding-aware C3 step (fused_c3.cu), bf16 tensor cores ----
+struct FusedC3 {
+  bool ready = false;                 // model side prepared (weights, T table)
+  const __nv_bfloat16* w1 = nullptr;  // aliases of the model's layer weights [N][K]
+  const __nv_bfloat16* w2 = nullptr;
+  const __nv_bfloat16* w3 = nullptr;
+  const __nv_bfloat16* wfc1 = nullptr;
+  const float *b1 = nullptr, *b2 = nullptr, *b3 = nullptr;
+  float* T = nullptr;                 // [15][256] constant fc1 table (owned)
+  const float* head_w = nullptr;      // fc2 [3][256]
+  const float* head_b = nullptr;
+  // per-run buffers (owned), sized for cap_n sub-traces
+  uint64_t cap_n = 0;
+  uint32_t* blocks = nullptr;         // [n*14] block ids b<<4|p
+  uint32_t* count = nullptr;          // [2] block counts by step parity
+  uint8_t* tileP[2] = {nullptr, nullptr};   // [ceil(n/128)] P_tile by step parity
+  __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
+  CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
+  CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
+};
+void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
+void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n, cudaStream_t st);
+void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
+                     cudaStream_t st);
+bool fused_make_maps(FusedC3& f, uint64_t n);
+bool fused_make_weight_maps(FusedC3& f);
+void fused_dump_debug();
 
 // pad/convert the caller's [B][112][50] fp32 inputs (psim_cnn_forward)
 void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st);

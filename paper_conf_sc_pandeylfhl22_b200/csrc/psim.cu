@@ -102,6 +102,7 @@ struct Prof {
 struct psim_ctx {
   psim_opts opts{};
   Prof prof;
+  FusedC3 fused;
   int cap = 110;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -218,6 +219,12 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->rec_lat);
   dfree(ctx->rec_k);
   dfree(ctx->rec_clock);
+  dfree(ctx->fused.T);
+  dfree(ctx->fused.blocks);
+  dfree(ctx->fused.count);
+  dfree(ctx->fused.tileP[0]);
+  dfree(ctx->fused.tileP[1]);
+  dfree(ctx->fused.a4);
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
@@ -393,6 +400,52 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
   m.arch = desc->arch;
   m.precision = ctx->opts.precision;
   m.loaded = true;
+  // fused padding-aware path (bf16 C3): constant table of the all-padding positions
+  FusedC3& fz = ctx->fused;
+  dfree(fz.T);
+  fz.T = nullptr;
+  fz.ready = false;
+  if (bf16 && desc->arch == PSIM_ARCH_C3) {
+    // c3 = conv3(conv2(conv1(0))) with the GPU's rounding points (bf16 operands,
+    // bias + ReLU, bf16 activations); T[P] = b_fc1 + sum_{p>=P} Wfc1[:, p*128:(p+1)*128] . c3
+    auto bf = [](double v) { uint16_t h = f32_to_bf16_rne((float)v); uint32_t u = (uint32_t)h << 16; float f; memcpy(&f, &u, 4); return (double)f; };
+    const float* W1 = w;              const float* B1 = W1 + 64 * 50 * 2;
+    const float* W2 = B1 + 64;        const float* B2 = W2 + 128 * 64 * 2;
+    const float* W3 = B2 + 128;       const float* B3 = W3 + 128 * 128 * 2;
+    const float* WF = B3 + 128;       const float* BF = WF + 256 * 1792;
+    (void)W1;
+    double r1[64], r2[128], c3[128];
+    for (int o = 0; o < 64; ++o) r1[o] = bf(std::max(0.0, (double)B1[o]));
+    for (int o = 0; o < 128; ++o) {
+      double acc = 0;
+      for (int c = 0; c < 64; ++c) for (int t = 0; t < 2; ++t) acc += bf(W2[(o * 64 + c) * 2 + t]) * r1[c];
+      r2[o] = bf(std::max(0.0, acc + B2[o]));
+    }
+    for (int o = 0; o < 128; ++o) {
+      double acc = 0;
+      for (int c = 0; c < 128; ++c) for (int t = 0; t < 2; ++t) acc += bf(W3[(o * 128 + c) * 2 + t]) * r2[c];
+      c3[o] = bf(std::max(0.0, acc + B3[o]));
+    }
+    std::vector<float> T(15 * 256);
+    for (int o = 0; o < 256; ++o) {
+      double acc = (double)BF[o];
+      T[14 * 256 + o] = (float)acc;
+      for (int P = 13; P >= 0; --P) {
+        for (int c = 0; c < 128; ++c) acc += bf(WF[(size_t)o * 1792 + P * 128 + c]) * c3[c];
+        T[P * 256 + o] = (float)acc;
+      }
+    }
+    CK(cudaMalloc(&fz.T, T.size() * 4));
+    CK(cudaMemcpy(fz.T, T.data(), T.size() * 4, cudaMemcpyHostToDevice));
+    fz.w1 = (const __nv_bfloat16*)m.layers[0].w; fz.b1 = m.layers[0].bias;
+    fz.w2 = (const __nv_bfloat16*)m.layers[1].w; fz.b2 = m.layers[1].bias;
+    fz.w3 = (const __nv_bfloat16*)m.layers[2].w; fz.b3 = m.layers[2].bias;
+    fz.wfc1 = (const __nv_bfloat16*)m.layers[3].w;
+    fz.head_w = m.head_w; fz.head_b = m.head_b;
+    if (!fused_make_weight_maps(fz)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for the conv weights");
+    fz.ready = true;
+    fz.cap_n = 0;   // per-run buffers and TMA maps are (re)made by simulate
+  }
   ctx->done = false;
   return PSIM_OK;
 }
@@ -527,7 +580,25 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
 
   int rc = ensure_state(ctx);
   if (rc) return rc;
-  if (predict) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
+  const bool fused = predict && ctx->fused.ready && !(ctx->opts.flags & PSIM_LAYERWISE) && (ctx->stride % 16) == 0;
+  if (predict && !fused) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
+  if (fused) {
+    FusedC3& fz = ctx->fused;
+    const uint64_t nn = std::max<uint64_t>(n, 1);
+    if (fz.cap_n != nn) {
+      dfree(fz.blocks); dfree(fz.count); dfree(fz.tileP[0]); dfree(fz.tileP[1]); dfree(fz.a4);
+      fz.blocks = nullptr; fz.count = nullptr; fz.tileP[0] = fz.tileP[1] = nullptr; fz.a4 = nullptr;
+      const uint64_t nt = (nn + 127) / 128;
+      CK(cudaMalloc(&fz.blocks, nn * 14 * 4));
+      CK(cudaMalloc(&fz.count, 16));
+      CK(cudaMalloc(&fz.tileP[0], nt + 16));
+      CK(cudaMalloc(&fz.tileP[1], nt + 16));
+      CK(cudaMalloc(&fz.a4, nn * 14 * 128 * 2));
+      CK(cudaMemset(fz.a4, 0, nn * 14 * 128 * 2));
+      if (!fused_make_maps(fz, nn)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for the fused path");
+      fz.cap_n = nn;
+    }
+  }
   const bool rec = (ctx->opts.flags & PSIM_RECORD_ROWS) != 0;
   if (rec && ctx->rec_cap < (size_t)rows) {
     dfree(ctx->rec_lat); dfree(ctx->rec_k); dfree(ctx->rec_clock);
@@ -575,7 +646,25 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
+  if (fused && n) {
+    // invariant of the fused path: a4 rows p >= P_b are zero (fc1 reads them as 0)
+    CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
+    pf.begin(PSIM_KC_OTHER);
+    launch_fused_init(ctx->fused, n, st);
+    pf.end(PSIM_KC_OTHER);
+  }
   for (int64_t t = 0; t < ctx->steps && n; ++t) {
+    if (fused) {
+      ga.step = t;
+      ua.step = t;
+      pf.begin(PSIM_KC_LAYER0);
+      launch_conv_stack(ctx->fused, ga, t, n, st);
+      pf.end(PSIM_KC_LAYER0);
+      pf.begin(PSIM_KC_LAYER0 + 3);
+      launch_fc1_head(ctx->fused, ua, ctx->st.e, t, forced, st);
+      pf.end(PSIM_KC_LAYER0 + 3);
+      continue;
+    }
     if (predict) {
       ga.step = t;
       pf.begin(PSIM_KC_GATHER);
@@ -621,7 +710,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   for (int c = 0; c < PSIM_KC_COUNT; ++c) { stats.kernel_launches[c] = pf.launches[c]; launches += pf.launches[c]; }
   stats.gpu_launches = launches;
   pf.collect(stats.kernel_ms);
-  for (size_t li = 0; li < ctx->model.layers.size() && li < 4 && predict; ++li) {
+  for (size_t li = 0; li < ctx->model.layers.size() && li < 4 && predict && !fused; ++li) {
     const GemmLayer& g = ctx->model.layers[li];
     stats.layer_m[li] = n * g.rows_per_item;
     stats.layer_n[li] = g.N;
@@ -637,6 +726,14 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     if (n) CK(cudaMemcpy(cyc.data(), ctx->st.cycles, n * 8, cudaMemcpyDeviceToHost));
     for (auto v : cyc) lc += v;
     stats.local_cycles = lc;
+  }
+  if (fused) fused_dump_debug();
+  if (fused) {   // GEMM shapes of the fused kernels: blocks (conv stack) and fc1 rows
+    uint64_t blocks = 0;
+    for (int k = 0; k < 112; ++k) blocks += stats.k_hist[k] * (uint64_t)((k + 8) / 8);
+    stats.layer_m[0] = blocks / std::max<uint64_t>(stats.steps, 1);   // mean blocks per step
+    stats.layer_n[0] = 128; stats.layer_k[0] = 0;
+    stats.layer_m[3] = n; stats.layer_n[3] = 256; stats.layer_k[3] = 0;
   }
   ctx->stats = stats;
   ctx->done = true;

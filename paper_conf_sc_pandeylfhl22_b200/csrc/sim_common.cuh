@@ -1,0 +1,211 @@
+// sim_common.cuh -- the integer queue update of one sub-trace, executed by one
+// warp (R3-R5, R7).  Shared by the standalone
+// update kernel (sim_kernels.cu) and the fused fc1/head/update kernel
+// (fused_c3.cu).  Product side only.
+#pragma once
+#include "internal.h"
+
+namespace psim {
+
+__device__ __forceinline__ int lat_round(float y) {
+  // R7: nearest integer, ties to even, on the fp32 value; NaN -> 0; clamp [0, 4095]
+  if (isnan(y)) return 0;
+  float r = rintf(y);
+  if (r < 0.f) return 0;
+  if (r > (float)kLatMax) return kLatMax;
+  return (int)r;
+}
+
+// Warp-cooperative update of sub-trace b at lockstep step a.step (caller has
+// checked the sub-trace is active).  y: the CNN's raw outputs (nullptr when
+// teacher-forced without prediction).  Returns the new context count (all lanes).
+// Lane l owns entries l, l+32, l+64, l+96 in registers; stable compaction by
+// ballot + popc keeps fetch order.
+__device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
+                                               int64_t nsteps, bool has_y, float y0, float y1, float y2,
+                                               int lane) {
+  const unsigned lt_mask = (1u << lane) - 1u;
+  const int64_t i = ws + a.step;
+  int f, c, s;                    // latencies that drive the update
+  int pf = 0, pc = 0, ps = 0;     // the CNN's rounded prediction (recorded)
+  if (has_y) { pf = lat_round(y0); pc = lat_round(y1); ps = lat_round(y2); }
+  if (a.forced) {
+    const uint16_t* p = a.forced + (i - a.row_lo) * 3;
+    f = p[0]; c = p[1]; s = p[2];
+    if (!has_y) { pf = f; pc = c; ps = s; }
+  } else {
+    f = pf; c = pc; s = ps;
+  }
+  int64_t clock = a.st.clock[b];
+  const int k = a.st.count[b];
+  const uint64_t qn = a.st.n;                            // entry stride (entry-major layout)
+  uint32_t* qs = a.st.q_seq + b;
+  uint32_t* qf = a.st.q_fetch + b;
+  uint32_t* qc = a.st.q_cs + b;
+
+  clock += f;
+  const uint32_t clo_push = (uint32_t)clock;
+  uint32_t eseq[4], efet[4], ecs[4];
+  bool valid[4];
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const int ent = lane + 32 * m;
+    valid[m] = ent < k;
+    if (valid[m]) { eseq[m] = qs[ent * qn]; efet[m] = qf[ent * qn]; ecs[m] = qc[ent * qn]; }
+    if (ent == k) {                                      // push the predicted instruction (R4)
+      valid[m] = true;
+      eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16);
+    }
+  }
+  __syncwarp();
+  // retire: keep iff retire > Clock  <=>  c + s - age > 0
+  auto live = [&](int m, uint32_t clo) -> bool {
+    if (!valid[m]) return false;
+    const int cs_sum = (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16);
+    return cs_sum - (int)(clo - efet[m]) > 0;
+  };
+  bool keep[4];
+  int kept = 0;
+  uint32_t clo = (uint32_t)clock;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
+  if (kept > a.cap) {                                    // ROB-full stall: Clock = min retire (R5)
+    int dmin = 0x7fffffff;
+#pragma unroll
+    for (int m = 0; m < 4; ++m)
+      if (keep[m]) dmin = min(dmin, (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16) - (int)(clo - efet[m]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) dmin = min(dmin, __shfl_xor_sync(0xffffffffu, dmin, o));
+    clock += dmin;
+    clo = (uint32_t)clock;
+    kept = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
+    if (lane == 0) atomicAdd(a.st.stalls, 1ull);
+  }
+  int base = 0;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const unsigned bal = __ballot_sync(0xffffffffu, keep[m]);
+    if (keep[m]) {
+      const uint64_t pos = (uint64_t)(base + __popc(bal & lt_mask)) * qn;
+      qs[pos] = eseq[m]; qf[pos] = efet[m]; qc[pos] = ecs[m];
+    }
+    base += __popc(bal);
+  }
+  if (lane == 0) {
+    a.st.count[b] = base;
+    a.st.clock[b] = clock;
+    int64_t bnd = a.st.bnd[b];
+    if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
+    if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
+    atomicAdd(a.st.k_hist + k, 1ull);
+    if (i >= s_b) {
+      const int64_t r = i - a.row_lo;
+      if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
+      if (a.rec_k) a.rec_k[r] = k;
+      if (a.rec_clock) a.rec_clock[r] = clock;
+    }
+  }
+  return base;
+}
+
+}  // namespace psim
+
+namespace psim {
+
+// Thread-per-sub-trace variant of the same update (used by the fused
+// fc1/head/update kernel, where one epilogue thread owns one sub-trace row of
+// the tile).  Streams the fetch-ordered entries with 16-byte loads and
+// compacts in place (write index <= read index); the rare ROB-full stall
+// (R5) re-filters the compacted entries once.  Returns the new count.
+// hist: per-CTA shared histogram of k (flushed by the caller).
+struct QBatch { uint32_t s[8], f[8], c[8]; };
+
+// first 8 entries of sub-trace b (entry-major layout), to be prefetched early
+__device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int k, QBatch& q) {
+  const uint64_t qn = st.n;
+#pragma unroll
+  for (int t = 0; t < 8; ++t)
+    if (t < k) { q.s[t] = st.q_seq[t * qn + b]; q.f[t] = st.q_fetch[t * qn + b]; q.c[t] = st.q_cs[t * qn + b]; }
+}
+
+__device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
+                                                      int64_t nsteps, int k, int64_t clock, const QBatch& first,
+                                                      bool has_y, float y0, float y1, float y2,
+                                                      unsigned int* hist) {
+  const int64_t i = ws + a.step;
+  int f, c, s;
+  int pf = 0, pc = 0, ps = 0;
+  if (has_y) { pf = lat_round(y0); pc = lat_round(y1); ps = lat_round(y2); }
+  if (a.forced) {
+    const uint16_t* p = a.forced + (i - a.row_lo) * 3;
+    f = p[0]; c = p[1]; s = p[2];
+    if (!has_y) { pf = f; pc = c; ps = s; }
+  } else {
+    f = pf; c = pc; s = ps;
+  }
+  const uint64_t qn = a.st.n;                              // entry-major: entry e at [e * n + b]
+  uint32_t* qs = a.st.q_seq + b;
+  uint32_t* qf = a.st.q_fetch + b;
+  uint32_t* qc = a.st.q_cs + b;
+  clock += f;
+  uint32_t clo = (uint32_t)clock;
+  // push the predicted instruction (R4) as entry k, then retire.
+  // Entries are streamed in batches of 8 with all loads of a batch in flight;
+  // consecutive threads (sub-traces) access consecutive words (coalesced).
+  const uint32_t push_s = (uint32_t)i, push_f = clo, push_c = (uint32_t)c | ((uint32_t)s << 16);
+  const int n_in = k + 1;
+  int w = 0;
+  int dmin = 0x7fffffff;   // min (retire - Clock) over kept entries
+  for (int e0 = 0; e0 < n_in; e0 += 8) {
+    uint32_t vs[8], vf[8], vc[8];
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+      const int e = e0 + t;
+      if (e < k) {
+        if (e0 == 0) { vs[t] = first.s[t]; vf[t] = first.f[t]; vc[t] = first.c[t]; }   // prefetched
+        else { vs[t] = qs[e * qn]; vf[t] = qf[e * qn]; vc[t] = qc[e * qn]; }
+      } else { vs[t] = push_s; vf[t] = push_f; vc[t] = push_c; }   // e == k: the pushed entry
+    }
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+      if (e0 + t >= n_in) break;
+      const int rem = (int)(vc[t] & 0xFFFF) + (int)(vc[t] >> 16) - (int)(clo - vf[t]);   // retire - Clock
+      if (rem > 0) {
+        const uint64_t o = (uint64_t)w * qn;
+        qs[o] = vs[t]; qf[o] = vf[t]; qc[o] = vc[t];
+        ++w;
+        dmin = min(dmin, rem);
+      }
+    }
+  }
+  if (w > a.cap) {                                         // ROB-full stall: Clock = min retire (R5)
+    clock += dmin;
+    clo = (uint32_t)clock;
+    const int n2 = w;
+    w = 0;
+    for (int e = 0; e < n2; ++e) {
+      const uint32_t sv = qs[e * qn], fv = qf[e * qn], cv = qc[e * qn];
+      if ((int)(cv & 0xFFFF) + (int)(cv >> 16) - (int)(clo - fv) > 0) {
+        qs[w * qn] = sv; qf[w * qn] = fv; qc[w * qn] = cv; ++w;
+      }
+    }
+    atomicAdd(a.st.stalls, 1ull);
+  }
+  a.st.count[b] = w;
+  a.st.clock[b] = clock;
+  int64_t bnd = a.st.bnd[b];
+  if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
+  if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
+  atomicAdd(hist + k, 1u);
+  if (i >= s_b) {
+    const int64_t r = i - a.row_lo;
+    if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
+    if (a.rec_k) a.rec_k[r] = k;
+    if (a.rec_clock) a.rec_clock[r] = clock;
+  }
+  return w;
+}
+
+}  // namespace psim

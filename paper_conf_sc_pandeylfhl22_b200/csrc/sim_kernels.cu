@@ -9,17 +9,9 @@
 // exactly from the low 32 bits of the clocks (q_fetch) whatever the absolute
 // Clock; the 65535 clamp of R7 is kept for completeness.
 #include "internal.h"
+#include "sim_common.cuh"
 
 namespace psim {
-
-__device__ __forceinline__ int lat_round(float y) {
-  // R7: nearest integer, ties to even, on the fp32 value; NaN -> 0; clamp [0, 4095]
-  if (isnan(y)) return 0;
-  float r = rintf(y);
-  if (r < 0.f) return 0;
-  if (r > (float)kLatMax) return kLatMax;
-  return (int)r;
-}
 
 template <typename T>
 __device__ __forceinline__ void store2(T* p, float a, float b);
@@ -29,7 +21,7 @@ __device__ __forceinline__ void store2<float>(float* p, float a, float b) {
 }
 template <>
 __device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
-  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);  // exact for |v| <= 256
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);  // RNE, as the oracle's bf16 mode
 }
 
 // X[b][r][c]: row 0 = current instruction (time columns 0), rows 1..k = live
@@ -48,9 +40,9 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
     const int k = a.count[b];
     const uint32_t clo = (uint32_t)a.clock[b];
     T* xb = x + b * (uint64_t)(kRows * kFeatPad);
-    const uint32_t* qs = a.q_seq + b * kQStride;
-    const uint32_t* qf = a.q_fetch + b * kQStride;
-    const uint32_t* qc = a.q_cs + b * kQStride;
+    const uint32_t* qs = a.q_seq + b;      // entry-major: entry e at [e * n]
+    const uint32_t* qf = a.q_fetch + b;
+    const uint32_t* qc = a.q_cs + b;
     for (int r = 0; r < kRows; ++r) {
       float v0 = 0.f, v1 = 0.f;
       if (r <= k) {
@@ -60,10 +52,10 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
           row = i;
         } else {
           const int ent = k - r;                                  // newest first
-          row = qs[ent];
-          const uint32_t cs = qc[ent];
+          row = qs[ent * a.n];
+          const uint32_t cs = qc[ent * a.n];
           const int c = cs & 0xFFFF, s = cs >> 16;
-          age = (int)(clo - qf[ent]);
+          age = (int)(clo - qf[ent * a.n]);
           remc = max(0, c - age);
           remr = c + s - age;
           age = min(age, kTimeMax); remc = min(remc, kTimeMax); remr = min(remr, kTimeMax);
@@ -105,98 +97,15 @@ void launch_gather_bf16(const GatherArgs& a, __nv_bfloat16* x, cudaStream_t st) 
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) update_kernel(UpdateArgs a) {
   const int lane = threadIdx.x & 31;
-  const unsigned lt_mask = (1u << lane) - 1u;
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
   for (uint64_t b = warp; b < a.st.n; b += nwarps) {
     const int64_t ws = a.st.ws[b], s_b = a.st.s[b], e_b = a.st.e[b];
     const int64_t nsteps = e_b - ws;
     if (a.step >= nsteps) continue;
-    const int64_t i = ws + a.step;
-    int f, c, s;          // latencies that drive the update
-    int pf = 0, pc = 0, ps = 0;   // the CNN's rounded prediction (recorded)
-    if (a.y) {
-      pf = lat_round(a.y[b * 3 + 0]);
-      pc = lat_round(a.y[b * 3 + 1]);
-      ps = lat_round(a.y[b * 3 + 2]);
-    }
-    if (a.forced) {
-      const uint16_t* p = a.forced + (i - a.row_lo) * 3;
-      f = p[0]; c = p[1]; s = p[2];
-      if (!a.y) { pf = f; pc = c; ps = s; }
-    } else {
-      f = pf; c = pc; s = ps;
-    }
-    int64_t clock = a.st.clock[b];
-    const int k = a.st.count[b];
-    uint32_t* qs = a.st.q_seq + b * kQStride;
-    uint32_t* qf = a.st.q_fetch + b * kQStride;
-    uint32_t* qc = a.st.q_cs + b * kQStride;
-
-    clock += f;
-    const uint32_t clo_push = (uint32_t)clock;
-    uint32_t eseq[4], efet[4], ecs[4];
-    bool valid[4];
-#pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      const int ent = lane + 32 * m;
-      valid[m] = ent < k;
-      if (valid[m]) { eseq[m] = qs[ent]; efet[m] = qf[ent]; ecs[m] = qc[ent]; }
-      if (ent == k) {                                      // push the predicted instruction (R4)
-        valid[m] = true;
-        eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16);
-      }
-    }
-    __syncwarp();
-    // retire: keep iff retire > Clock  <=>  c + s - age > 0
-    auto live = [&](int m, uint32_t clo) -> bool {
-      if (!valid[m]) return false;
-      const int cs_sum = (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16);
-      return cs_sum - (int)(clo - efet[m]) > 0;
-    };
-    bool keep[4];
-    int kept = 0;
-    uint32_t clo = (uint32_t)clock;
-#pragma unroll
-    for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
-    if (kept > a.cap) {                                    // ROB-full stall: Clock = min retire (R5)
-      int dmin = 0x7fffffff;
-#pragma unroll
-      for (int m = 0; m < 4; ++m)
-        if (keep[m]) dmin = min(dmin, (int)(ecs[m] & 0xFFFF) + (int)(ecs[m] >> 16) - (int)(clo - efet[m]));
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) dmin = min(dmin, __shfl_xor_sync(0xffffffffu, dmin, o));
-      clock += dmin;
-      clo = (uint32_t)clock;
-      kept = 0;
-#pragma unroll
-      for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
-      if (lane == 0) atomicAdd(a.st.stalls, 1ull);
-    }
-    int base = 0;
-#pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      const unsigned bal = __ballot_sync(0xffffffffu, keep[m]);
-      if (keep[m]) {
-        const int pos = base + __popc(bal & lt_mask);
-        qs[pos] = eseq[m]; qf[pos] = efet[m]; qc[pos] = ecs[m];
-      }
-      base += __popc(bal);
-    }
-    if (lane == 0) {
-      a.st.count[b] = base;
-      a.st.clock[b] = clock;
-      int64_t bnd = a.st.bnd[b];
-      if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
-      if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
-      atomicAdd(a.st.k_hist + k, 1ull);
-      if (i >= s_b) {
-        const int64_t r = i - a.row_lo;
-        if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
-        if (a.rec_k) a.rec_k[r] = k;
-        if (a.rec_clock) a.rec_clock[r] = clock;
-      }
-    }
+    const bool has_y = a.y != nullptr;
+    update_subtrace(a, b, ws, s_b, nsteps, has_y, has_y ? a.y[b * 3] : 0.f, has_y ? a.y[b * 3 + 1] : 0.f,
+                    has_y ? a.y[b * 3 + 2] : 0.f, lane);
   }
 }
 

@@ -23,9 +23,9 @@ pytestmark = pytest.mark.gpu
 
 
 def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, forced=None,
-            record=True, rank=0, world=1, first_row=0, n_instr=None, device_trace=False):
+            record=True, rank=0, world=1, first_row=0, n_instr=None, device_trace=False, layerwise=False):
     with P.Simulator(precision=precision, queue_cap=cap, record_rows=record, rank=rank,
-                     world_size=world) as sim:
+                     world_size=world, layerwise=layerwise) as sim:
         if device_trace:
             t = torch.from_numpy(np.ascontiguousarray(trace)).cuda()
             sim.load_trace(t, n_instr=n_instr, first_row=first_row)
@@ -193,7 +193,7 @@ def test_s2_cnn_bf16_tensor_cores(arch):
 # So S3 is split: (a) decision agreement -- the GPU's gather + CNN + rounding on
 # the ORACLE's trajectory (teacher-forced queue, PSIM_FORCE_PREDICT) must agree
 # on >= 99.9% of per-instruction (f, c, s); (b) free-running totals within 0.5%.
-def decision_parity(tr, N, arch, w, precision, samples=None, cap=110):
+def decision_parity(tr, N, arch, w, precision, samples=None, cap=110, layerwise=False):
     """W = 0 so the per-row forced latencies are exactly each sub-trace's oracle trajectory."""
     L = tr.shape[0]
     mode = oracle.BF16 if precision == "bf16" else oracle.FP64
@@ -205,7 +205,8 @@ def decision_parity(tr, N, arch, w, precision, samples=None, cap=110):
         s, e = j * L // N, (j + 1) * L // N
         forced[s:e] = ref["lat"][s:e]
         rows.append((s, e))
-    with P.Simulator(precision=precision, record_rows=True, force_predict=True, queue_cap=cap) as sim:
+    with P.Simulator(precision=precision, record_rows=True, force_predict=True, queue_cap=cap,
+                     layerwise=layerwise) as sim:
         sim.load_trace(tr)
         sim.partition(N, 0)
         sim.load_model(arch, w)
@@ -219,10 +220,10 @@ def decision_parity(tr, N, arch, w, precision, samples=None, cap=110):
     return agree / n
 
 
-def free_running(tr, N, W, arch, w, precision, samples=None):
+def free_running(tr, N, W, arch, w, precision, samples=None, layerwise=False):
     L = tr.shape[0]
     mode = oracle.BF16 if precision == "bf16" else oracle.FP64
-    g = gpu_run(tr, N, W, arch=arch, weights=w, precision=precision)
+    g = gpu_run(tr, N, W, arch=arch, weights=w, precision=precision, layerwise=layerwise)
     js = list(range(N)) if samples is None else list(samples)
     ref_c, gpu_c, agree, n = 0, 0, 0, 0
     for j in js:
@@ -244,14 +245,58 @@ def test_s3_config1_m2_fp32():
     assert rel <= 0.005
 
 
-@pytest.mark.parametrize("precision", ["bf16", "fp32"])
-def test_s3_c3_small(precision):
+@pytest.mark.parametrize("precision,layerwise", [("bf16", False), ("bf16", True), ("fp32", False)])
+def test_s3_c3_small(precision, layerwise):
+    """bf16 runs the fused padding-aware kernels by default (layerwise=False) and the
+    layer-by-layer tcgen05 GEMMs with layerwise=True; fp32 runs the SIMT path."""
     L, N = 3000, 6
     tr = synth.trace(L, 2024)
     w = synth.weights("C3")
-    assert decision_parity(tr, N, "C3", w, precision) >= 0.999
-    rel, agree, _ = free_running(tr, N, 64, "C3", w, precision)
+    assert decision_parity(tr, N, "C3", w, precision, layerwise=layerwise) >= 0.999
+    rel, agree, _ = free_running(tr, N, 64, "C3", w, precision, layerwise=layerwise)
     assert rel <= 0.005, (rel, agree)
+
+
+def test_s3_fused_full_queue_and_ragged_tiles():
+    """Fused path: contexts filled to the 110-entry cap (all 14 conv3 positions
+    computed, P = 14) by long completion latencies, ragged sub-trace counts
+    (N = 300: tiles of 128 + a partial tile) and finished sub-traces (ragged lengths)."""
+    L, N = 45_017, 300                      # ~150 instructions per sub-trace, ragged
+    tr = synth.trace(L, 99)
+    w = synth.weights("C3")
+    forced = synth.teacher_latencies(L, 23, c_mean=400.0)        # queues saturate: k -> 110, stalls
+    mode = oracle.BF16
+    refs = {}
+    for j in (0, 7, 128, 255, 299):
+        ref = oracle.simulate(tr, N, 0, forced_lat=forced, j0=j, nj=1, cap=110)
+        refs[j] = ref
+    # decision agreement of the CNN on those saturated trajectories
+    with P.Simulator(precision="bf16", record_rows=True, force_predict=True) as sim:
+        sim.load_trace(tr); sim.partition(N, 0); sim.load_model("C3", w); sim.force_latencies(forced)
+        sim.simulate()
+        st = sim.stats()
+        assert max(i for i, c in enumerate(st["k_hist"]) if c) == 110
+        agree, legit, n, bad = 0, 0, 0, []
+        for j in refs:
+            s, e = j * L // N, (j + 1) * L // N
+            lat, k, clk = sim.get_rows(s, e - s)
+            assert np.array_equal(k, refs[j]["k"][s:e]) and np.array_equal(clk, refs[j]["clock"][s:e])
+            q = oracle.Queue(110)
+            for i in range(s, e):            # the oracle's own CNN decision on the same state
+                X, kk = q.build_input(tr, i)
+                y = oracle.cnn_forward("C3", w, X, mode=mode)
+                ref = tuple(oracle.round_latency(v) for v in y)
+                got = tuple(int(v) for v in lat[i - s])
+                n += 1
+                if ref == got:
+                    agree += 1
+                elif all(r == g or abs(abs(v - np.floor(v)) - 0.5) <= 1e-3 * max(abs(v), 1.0)
+                         for r, g, v in zip(ref, got, y)):
+                    legit += 1                   # R15: within S2's tolerance of a .5 boundary
+                else:
+                    bad.append((i, kk, ref, got, y))
+                q.update(i, *(int(v) for v in forced[i]))
+        assert not bad and (agree + legit) / n >= 0.999 and agree / n >= 0.99, (agree, legit, n, bad[:5])
 
 
 def test_s3_config2_full_size_sampled():
