@@ -107,14 +107,14 @@ def roofline(stats, k_steps, cfg):
     avg_s = ms[dom] / 1e3 / max(launches[dom], 1)
     hist = np.array(stats["k_hist"], np.float64)
     kmean = float((hist * np.arange(112)).sum() / max(hist.sum(), 1))
-    fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0
+    fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0   # fused path: conv_stack + fc1_head
     if names[dom].startswith("gemm_layer"):
         li = int(names[dom][-1])
         M, N, K = stats["layer_m"][li], stats["layer_n"][li], stats["layer_k"][li]
         if fused and li == 0:     # conv_stack: per (sub-trace, position) block conv1 4x2x100x64 + conv2 2x2x128x128 + conv3 2x256x128
             flops = float(M) * 247808.0
-        elif fused and li == 3:   # fc1 over P_tile positions (tile max of P_b), N = 256
-            flops = 2.0 * M * 256 * 128 * stats.get("mean_ptile", 5.0)
+        elif fused and li == 3:   # fc1 over P_tile positions (tile max of P_b): K = 128 * mean P_tile
+            flops = 2.0 * M * 256 * (stats["layer_k"][3] / 1000.0)
         else:
             k_alg = 100 if li == 0 else K      # conv1: 2 rows x 50 real features (features padded to 64)
             flops = 2.0 * M * N * k_alg
@@ -225,7 +225,7 @@ def main():
         val = insts / tot / 1e6
         line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "MIPS", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
-                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64" if cfg["precision"] == "fp32" else "f64 (bf16 operand rounding)",
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic", "config": config,
                 "cpu_baseline": {"value": val, "unit": "MIPS", "cores": 1, "kind": "oracle",
                                  "sample": f"{insts} instructions of whole random sub-traces of {args.config} per "

@@ -24,7 +24,7 @@ BUILD = os.path.join(PKG, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-I", INCLUDE, "-I", CSRC,
-                "--expt-relaxed-constexpr", "-Xptxas", "-v"]
+                "--expt-relaxed-constexpr", "-Xptxas", "-v"] + (["-DPSIM_TIMING"] if os.environ.get("PSIM_TIMING") else [])
 
 
 def _sources():

@@ -75,11 +75,18 @@ struct ConvArgs {
   long long* dbg;            // optional stage timestamps of CTA 0 (PSIM_DEBUG_TIMING), else nullptr
 };
 
-// debug timestamps: dbg[tile * 256 + slot] = clock64() for CTA 0, first 4 tiles
+// debug timestamps (build with PSIM_TIMING=1): dbg[tile * 256 + slot] = clock64()
+// for CTA 0, first 4 tiles of the step named by $PSIM_DEBUG_TIMING
+#ifdef PSIM_TIMING
 #define PSIM_TS(slot)                                                                                   \
   do {                                                                                                 \
     if (a.dbg && blockIdx.x == 0 && it < 4 && lane == 0) a.dbg[it * 256 + (slot)] = clock64();        \
   } while (0)
+#else
+#define PSIM_TS(slot) \
+  do {                \
+  } while (0)
+#endif
 
 __device__ __forceinline__ uint32_t bf16_bits_u8(uint32_t v) {   // exact: v < 256
   return __float_as_uint((float)v) >> 16;
@@ -480,6 +487,7 @@ struct HeadArgs {
   const float* b2;           // [3]
   int force_predict;         // run the head even when teacher-forced
   long long* dbg;            // optional timestamps (PSIM_DEBUG_TIMING), slots 128..
+  unsigned long long* ptile_sum;   // sum of P_tile over the tiles of the run (fc1 K statistics)
 };
 
 __global__ void __launch_bounds__(fh::THREADS, 1)
@@ -629,6 +637,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const int yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const bool inb = b < n;
+      const int tileP_cur = a.tileP[tt];
       int64_t ws = 0, s_b = 0, nsteps = 0, clock = 0;
       int kb = 0;
       if (inb) {   // prefetch the state and the first queue entries while the head runs
@@ -675,7 +684,9 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       if (m == 0) {
         const int total = sPg[0] + sPg[1] + sPg[2] + sPg[3];
         sPg[8] = total ? (int)atomicAdd(a.next_count, (uint32_t)total) : 0;
-        a.tileP_next[tt] = (uint8_t)max(max(sPg[4], sPg[5]), max(sPg[6], sPg[7]));
+        const int ptn = max(max(sPg[4], sPg[5]), max(sPg[6], sPg[7]));
+        a.tileP_next[tt] = (uint8_t)ptn;
+        if (a.ptile_sum && tileP_cur > 0) atomicAdd(a.ptile_sum, (unsigned long long)tileP_cur);
       }
       named_bar_sync(2 + grp, 128);
       const uint32_t base = (uint32_t)sPg[8] + (uint32_t)(before + incl - pnext);
@@ -816,6 +827,7 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
   a.T = f.T; a.w2 = f.head_w; a.b2 = f.head_b;
   a.force_predict = force_predict ? 1 : 0;
   a.dbg = debug_buffer(step);
+  a.ptile_sum = u.st.ptile_sum;
   const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
   const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
   fc1_head_kernel<<<grid, fh::THREADS, fh::SMEM, st>>>(f.mapA, f.mapB, a);

@@ -62,6 +62,7 @@ struct SimState {
   uint32_t* q_cs = nullptr;     // [kQStride][n] c | s << 16
   unsigned long long* k_hist = nullptr;   // [112]
   unsigned long long* stalls = nullptr;   // [1]
+  unsigned long long* ptile_sum = nullptr;   // [1] fused fc1: sum of P_tile over tiles and steps
   long long* total = nullptr;             // [1] local sum of cycles (NCCL send/recv buffer)
 };
 

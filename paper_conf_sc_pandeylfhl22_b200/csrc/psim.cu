@@ -210,7 +210,7 @@ void psim_destroy(psim_ctx* ctx) {
   SimState& s = ctx->st;
   for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
                   (void*)s.count, (void*)s.q_seq, (void*)s.q_fetch, (void*)s.q_cs, (void*)s.k_hist,
-                  (void*)s.stalls, (void*)s.total})
+                  (void*)s.stalls, (void*)s.total, (void*)s.ptile_sum})
     dfree(p);
   dfree(ctx->buf.x);
   for (void* p : ctx->buf.act) dfree(p);
@@ -551,6 +551,7 @@ static int ensure_state(psim_ctx* ctx) {
     CK(cudaMalloc(&s.k_hist, 112 * 8));
     CK(cudaMalloc(&s.stalls, 8));
     CK(cudaMalloc(&s.total, 8));
+    CK(cudaMalloc(&s.ptile_sum, 8));
   }
   s.n = n;
   if (n) {
@@ -690,9 +691,10 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   CK(cudaEventRecord(ctx->ev[2], st));
   long long total = 0;
   CK(cudaMemcpyAsync(&total, ctx->st.total, 8, cudaMemcpyDeviceToHost, st));
-  unsigned long long hist[112], stalls = 0;
+  unsigned long long hist[112], stalls = 0, ptile_sum = 0;
   CK(cudaMemcpyAsync(hist, ctx->st.k_hist, sizeof hist, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(&stalls, ctx->st.stalls, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&ptile_sum, ctx->st.ptile_sum, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   CK(cudaGetLastError());
   float ms_all = 0, ms_load = 0;
@@ -733,7 +735,10 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     for (int k = 0; k < 112; ++k) blocks += stats.k_hist[k] * (uint64_t)((k + 8) / 8);
     stats.layer_m[0] = blocks / std::max<uint64_t>(stats.steps, 1);   // mean blocks per step
     stats.layer_n[0] = 128; stats.layer_k[0] = 0;
-    stats.layer_m[3] = n; stats.layer_n[3] = 256; stats.layer_k[3] = 0;
+    // fc1: M = sub-traces, N = 256, K = 128 x (mean P_tile over tiles), reported x1000 in layer_k
+    const uint64_t tiles = ((n + 127) / 128) * std::max<uint64_t>(stats.steps, 1);
+    stats.layer_m[3] = n; stats.layer_n[3] = 256;
+    stats.layer_k[3] = (uint32_t)(1000.0 * 128.0 * (double)ptile_sum / (double)tiles);
   }
   ctx->stats = stats;
   ctx->done = true;

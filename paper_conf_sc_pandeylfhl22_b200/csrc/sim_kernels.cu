@@ -117,7 +117,7 @@ __global__ void state_init_kernel(SimState s) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (t < s.n) { s.clock[t] = 0; s.bnd[t] = 0; s.cycles[t] = 0; s.count[t] = 0; }
   if (t < 112) s.k_hist[t] = 0;
-  if (t == 0) { *s.stalls = 0; *s.total = 0; }
+  if (t == 0) { *s.stalls = 0; *s.total = 0; *s.ptile_sum = 0; }
 }
 void launch_state_init(const SimState& s, cudaStream_t st) {
   uint64_t n = s.n > 112 ? s.n : 112;
