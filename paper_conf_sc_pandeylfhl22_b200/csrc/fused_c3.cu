@@ -46,9 +46,9 @@ constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
 constexpr int BAR_OFF = A3_OFF + 32 * 1024;  // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 256;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
-constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 256, TMEM_COLS = 512;
-constexpr int THREADS = 448;   // warps 0-3 epilogue, 4 MMA, 5-12 gather, 13 a4 write-back
-constexpr int MMA_WARP = 4, GATHER_WARP0 = 5, WB_WARP = 13;
+constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
+constexpr int THREADS = 448;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi), 8 MMA, 9-12 gather, 13 write-back
+constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, WB_WARP = 13;
 }  // namespace cs
 
 struct ConvArgs {
@@ -113,22 +113,22 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
-  uint64_t* xfull = bars + 0;    // [2]  8 gather warps
-  uint64_t* xempty = bars + 2;   // [2]  commit
-  uint64_t* c1full = bars + 4;   // [2]  commit
-  uint64_t* c1empty = bars + 6;  // [2]  4 epilogue warps
-  uint64_t* a2full = bars + 8;   //      4
-  uint64_t* a2empty = bars + 9;  //      commit
-  uint64_t* c2full = bars + 10;  //      commit
-  uint64_t* c2empty = bars + 11; //      4
-  uint64_t* a3full = bars + 12;  //      4
-  uint64_t* a3empty = bars + 13; //      commit
-  uint64_t* c3full = bars + 14;  //      commit
-  uint64_t* c3empty = bars + 15; //      4
-  uint64_t* wbar = bars + 16;    //      weights landed (TMA)
-  uint64_t* stg_full = bars + 17;   //   4: conv3 rows staged in the A3 region
-  uint64_t* stg_empty = bars + 18;  //   1: write-back warp done reading the staging rows
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 19);
+  uint64_t* xfull = bars + 0;      // [2] 4 gather warps
+  uint64_t* xempty = bars + 2;     // [2] commit
+  uint64_t* c1full = bars + 4;     // [2] commit
+  uint64_t* c1empty = bars + 6;    // [2] 4 (EG-A)
+  uint64_t* a2full = bars + 8;     //     4 (EG-A)
+  uint64_t* a2empty = bars + 9;    //     commit
+  uint64_t* c2full = bars + 10;    // [2] commit (one TMEM slot per conv2 position)
+  uint64_t* c2empty = bars + 12;   // [2] 4 (EG-B)
+  uint64_t* a3full = bars + 14;    //     4 (EG-B)
+  uint64_t* a3empty = bars + 15;   //     commit
+  uint64_t* c3full = bars + 16;    //     commit
+  uint64_t* c3empty = bars + 17;   //     4 (EG-B)
+  uint64_t* wbar = bars + 18;      //     weights + biases landed
+  uint64_t* stg_full = bars + 19;  //     4 (EG-B): conv3 rows staged in the A3 region
+  uint64_t* stg_empty = bars + 20; //     1 (write-back warp)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 21);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t nblocks = *a.nblocks;
@@ -137,10 +137,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
 
   if (tid == 0) {
     for (int i = 0; i < 2; ++i) {
-      mbar_init(xfull + i, 8); mbar_init(xempty + i, 1);
+      mbar_init(xfull + i, 4); mbar_init(xempty + i, 1);
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
+      mbar_init(c2full + i, 1); mbar_init(c2empty + i, 4);
     }
-    mbar_init(a2full, 4); mbar_init(a2empty, 1); mbar_init(c2full, 1); mbar_init(c2empty, 4);
+    mbar_init(a2full, 4); mbar_init(a2empty, 1);
     mbar_init(a3full, 4); mbar_init(a3empty, 1); mbar_init(c3full, 1); mbar_init(c3empty, 4);
     mbar_init(wbar, 1);
     mbar_init(stg_full, 4); mbar_init(stg_empty, 1);
@@ -167,65 +168,69 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
 
   if (warp == cs::MMA_WARP) {
     if (lane == 0) {   // ============================ MMA issuer
+      // Per tile: c1(0) c1(1) [c3 of the previous tile, K-half 1] c2(0,*) c1(2) c1(3) c3(0) c2(1,*);
+      // deferring the previous tile's last conv3 MMA lets this tile's conv1 overlap its epilogues.
       const uint32_t sbase = smem_u32(sm);
       const uint32_t id64 = idesc_bf16(128, 64), id128 = idesc_bf16(128, 128);
+      auto c1 = [&](uint32_t it, int j) {
+        const int s = j & 1;
+        const uint32_t n = it * 2 + (j >> 1);
+        PSIM_TS(0 + 2 * j);
+        wait_full(xfull + s, n);
+        wait_empty(c1empty + s, n);
+        PSIM_TS(1 + 2 * j);
+        fence_after();
+        const uint32_t xa = sbase + cs::X_OFF + s * 32768;
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
+                   sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
+        mma_commit(xempty + s);
+        mma_commit(c1full + s);
+      };
+      auto c2 = [&](uint32_t it, int h, int kh) {
+        PSIM_TS(8 + 2 * (h * 2 + kh));
+        wait_full(a2full, it * 4 + h * 2 + kh);
+        if (kh == 0) wait_empty(c2empty + h, it);
+        PSIM_TS(9 + 2 * (h * 2 + kh));
+        fence_after();
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          mma_bf16(tmem + cs::TMEM_C2 + h * 128, sw128_desc(sbase + cs::A2_OFF + k * 32),
+                   sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
+        mma_commit(a2empty);
+        if (kh == 1) mma_commit(c2full + h);
+      };
+      auto c3 = [&](uint32_t it, int kh) {
+        PSIM_TS(16 + 2 * kh);
+        wait_full(a3full, it * 2 + kh);
+        if (kh == 0) wait_empty(c3empty, it);
+        PSIM_TS(17 + 2 * kh);
+        fence_after();
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          mma_bf16(tmem + cs::TMEM_C3, sw128_desc(sbase + cs::A3_OFF + (k >> 2) * 16384 + (k & 3) * 32),
+                   sw128_desc(sbase + cs::W3_OFF + (2 * kh + (k >> 2)) * 16384 + (k & 3) * 32), id128,
+                   (kh | k) != 0);
+        mma_commit(a3empty);
+        if (kh == 1) mma_commit(c3full);
+      };
       uint32_t it = 0;
       for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
-        auto c1 = [&](int j) {
-          const int s = j & 1;
-          const uint32_t n = it * 2 + (j >> 1);
-          PSIM_TS(0 + 2 * j);
-          wait_full(xfull + s, n);
-          wait_empty(c1empty + s, n);
-          PSIM_TS(1 + 2 * j);
-          fence_after();
-          const uint32_t xa = sbase + cs::X_OFF + s * 32768;
-#pragma unroll
-          for (int k = 0; k < 8; ++k)
-            mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
-                     sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
-          mma_commit(xempty + s);
-          mma_commit(c1full + s);
-        };
-        auto c2 = [&](int h, int kh) {
-          const uint32_t n = it * 4 + h * 2 + kh;
-          PSIM_TS(8 + 2 * (h * 2 + kh));
-          wait_full(a2full, n);
-          if (kh == 0) wait_empty(c2empty, it * 2 + h);
-          PSIM_TS(9 + 2 * (h * 2 + kh));
-          fence_after();
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            mma_bf16(tmem + cs::TMEM_C2, sw128_desc(sbase + cs::A2_OFF + k * 32),
-                     sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
-          mma_commit(a2empty);
-          if (kh == 1) mma_commit(c2full);
-        };
-        auto c3 = [&](int kh) {
-          PSIM_TS(16 + 2 * kh);
-          wait_full(a3full, it * 2 + kh);
-          if (kh == 0) wait_empty(c3empty, it);
-          PSIM_TS(17 + 2 * kh);
-          fence_after();
-#pragma unroll
-          for (int k = 0; k < 8; ++k)
-            mma_bf16(tmem + cs::TMEM_C3, sw128_desc(sbase + cs::A3_OFF + (k >> 2) * 16384 + (k & 3) * 32),
-                     sw128_desc(sbase + cs::W3_OFF + (2 * kh + (k >> 2)) * 16384 + (k & 3) * 32), id128,
-                     (kh | k) != 0);
-          mma_commit(a3empty);
-          if (kh == 1) mma_commit(c3full);
-        };
-        c1(0); c1(1); c2(0, 0); c2(0, 1); c1(2); c1(3); c3(0); c2(1, 0); c2(1, 1); c3(1);
-        PSIM_TS(20);
+        c1(it, 0); c1(it, 1);
+        if (it > 0) c3(it - 1, 1);
+        c2(it, 0, 0); c2(it, 0, 1); c1(it, 2); c1(it, 3); c3(it, 0); c2(it, 1, 0); c2(it, 1, 1);
       }
+      if (it > 0) c3(it - 1, 1);
     }
-  } else if (warp < 4) {   // ============================ epilogues
+  } else if (warp < 4) {   // ============================ EG-A: conv1 epilogues (C1 -> A2)
     const int q = warp & 3;
     const int m = q * 32 + lane;                    // tile row = TMEM lane
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t it = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
-      auto e1 = [&](int j) {   // C1 (64 fp32) -> relu(+b1) -> bf16 -> A2
+#pragma unroll 1
+      for (int j = 0; j < 4; ++j) {
         const int s = j & 1;
         if (q == 0) PSIM_TS(32 + 4 * j);
         wait_full(c1full + s, it * 2 + (j >> 1));
@@ -258,88 +263,90 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(a2full);
         if (q == 0) PSIM_TS(48 + j);
-      };
-      auto e2 = [&](int h) {   // C2 (128 fp32) -> relu(+b2) -> bf16 -> A3 (2 atoms)
+      }
+    }
+  } else if (warp < 8) {   // ============================ EG-B: conv2 / conv3 epilogues
+    const int q = warp & 3;
+    const int m = q * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(q * 32) << 16;
+    uint32_t it = 0;
+    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (2 atoms)
         if (q == 0) PSIM_TS(56 + 4 * h);
-        wait_full(c2full, it * 2 + h);
+        wait_full(c2full + h, it);
         if (q == 0) PSIM_TS(57 + 4 * h);
         fence_after();
         wait_empty(a3empty, it * 2 + h);
         if (h == 0) wait_empty(stg_empty, it);        // previous tile's staging rows written back
         if (q == 0) PSIM_TS(58 + 4 * h);
 #pragma unroll 1
-        for (int cp = 0; cp < 2; ++cp) {              // 2 x (two TMEM loads in flight, one wait)
+        for (int cp = 0; cp < 2; ++cp) {
           uint32_t r0[32], r1[32];
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + cp * 64, r0);
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + cp * 64 + 32, r1);
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
+          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
           tmem_wait_ld();
-          uint32_t pk[32];
-#pragma unroll
-          for (int c = 0; c < 16; ++c) {
-            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb2[cp * 64 + 2 * c], 0.f),
-                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb2[cp * 64 + 2 * c + 1], 0.f));
-            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb2[cp * 64 + 32 + 2 * c], 0.f),
-                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb2[cp * 64 + 33 + 2 * c], 0.f));
-          }
           uint8_t* atom = sm + cs::A3_OFF + cp * 16384;   // 64 channels per atom
 #pragma unroll
-          for (int c = 0; c < 8; ++c)
-            st_sw128(atom, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
+          for (int c = 0; c < 4; ++c)
+            st_sw128(atom, m, c, make_uint4(
+                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 0]) + sb2[cp * 64 + 8 * c + 0], 0.f), fmaxf(__uint_as_float(r0[8 * c + 1]) + sb2[cp * 64 + 8 * c + 1], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 2]) + sb2[cp * 64 + 8 * c + 2], 0.f), fmaxf(__uint_as_float(r0[8 * c + 3]) + sb2[cp * 64 + 8 * c + 3], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 4]) + sb2[cp * 64 + 8 * c + 4], 0.f), fmaxf(__uint_as_float(r0[8 * c + 5]) + sb2[cp * 64 + 8 * c + 5], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 6]) + sb2[cp * 64 + 8 * c + 6], 0.f), fmaxf(__uint_as_float(r0[8 * c + 7]) + sb2[cp * 64 + 8 * c + 7], 0.f))));
+#pragma unroll
+          for (int c = 0; c < 4; ++c)
+            st_sw128(atom, m, 4 + c, make_uint4(
+                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 0]) + sb2[cp * 64 + 32 + 8 * c + 0], 0.f), fmaxf(__uint_as_float(r1[8 * c + 1]) + sb2[cp * 64 + 32 + 8 * c + 1], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 2]) + sb2[cp * 64 + 32 + 8 * c + 2], 0.f), fmaxf(__uint_as_float(r1[8 * c + 3]) + sb2[cp * 64 + 32 + 8 * c + 3], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 4]) + sb2[cp * 64 + 32 + 8 * c + 4], 0.f), fmaxf(__uint_as_float(r1[8 * c + 5]) + sb2[cp * 64 + 32 + 8 * c + 5], 0.f)),
+                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 6]) + sb2[cp * 64 + 32 + 8 * c + 6], 0.f), fmaxf(__uint_as_float(r1[8 * c + 7]) + sb2[cp * 64 + 32 + 8 * c + 7], 0.f))));
         }
         fence_before();
         fence_async_smem();
         __syncwarp();
-        if (lane == 0) { mbar_arrive(c2empty); mbar_arrive(a3full); }
+        if (lane == 0) { mbar_arrive(c2empty + h); mbar_arrive(a3full); }
         if (q == 0) PSIM_TS(59 + 4 * h);
-      };
-      auto e3 = [&]() {        // C3 (128 fp32) -> relu(+b3) -> bf16 -> A3 staging rows -> write-back warp
-        if (q == 0) PSIM_TS(64);
-        wait_full(c3full, it);   // c3 done: A3 is free for staging
-        if (q == 0) PSIM_TS(65);
-        fence_after();
-        uint8_t* row = sm + cs::A3_OFF + m * 256;     // plain row-major staging [128][256 B]
-#pragma unroll 1
-        for (int cp = 0; cp < 2; ++cp) {
-          uint32_t r0[32], r1[32];
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64, r0);
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64 + 32, r1);
-          tmem_wait_ld();
-          uint32_t pk[32];
-#pragma unroll
-          for (int c = 0; c < 16; ++c) {
-            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb3[cp * 64 + 2 * c], 0.f),
-                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb3[cp * 64 + 2 * c + 1], 0.f));
-            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb3[cp * 64 + 32 + 2 * c], 0.f),
-                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb3[cp * 64 + 33 + 2 * c], 0.f));
-          }
-#pragma unroll
-          for (int c = 0; c < 8; ++c) {   // lane-rotated chunk order: conflict-free 256-B row pitch
-            const int sel = (c + m) & 7;
-            uint4 v = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-#pragma unroll
-            for (int t = 1; t < 8; ++t)
-              if (sel == t) v = make_uint4(pk[4 * t], pk[4 * t + 1], pk[4 * t + 2], pk[4 * t + 3]);
-            *reinterpret_cast<uint4*>(row + (cp * 8 + sel) * 16) = v;
-          }
-          if (q == 0) PSIM_TS(67 + cp);
-        }
-        fence_before();
-        fence_async_smem();                           // staging rows are read by TMA bulk copies
-        __syncwarp();
-        if (lane == 0) { mbar_arrive(c3empty); mbar_arrive(stg_full); }
-        if (q == 0) PSIM_TS(66);
-      };
-      // same order as the MMA issue schedule: e1(0) e1(1) e2(0) e1(2) e1(3) e2(1) e3
-#pragma unroll 1
-      for (int ev = 0; ev < 7; ++ev) {
-        if (ev == 2 || ev == 5) e2(ev == 5);
-        else if (ev == 6) e3();
-        else e1(ev < 2 ? ev : ev - 1);
       }
+      // C3 (128 fp32) -> relu(+b3) -> bf16 -> plain staging rows in the A3 region -> write-back warp
+      if (q == 0) PSIM_TS(64);
+      wait_full(c3full, it);                          // conv3 done: A3 is free for staging
+      if (q == 0) PSIM_TS(65);
+      fence_after();
+      uint8_t* row = sm + cs::A3_OFF + m * 256;
+#pragma unroll 1
+      for (int cp = 0; cp < 2; ++cp) {
+        uint32_t r0[32], r1[32];
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64 + 32, r1);
+        tmem_wait_ld();
+        uint32_t pk[32];
+#pragma unroll
+        for (int c = 0; c < 16; ++c) {
+          pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb3[cp * 64 + 2 * c], 0.f),
+                            fmaxf(__uint_as_float(r0[2 * c + 1]) + sb3[cp * 64 + 2 * c + 1], 0.f));
+          pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb3[cp * 64 + 32 + 2 * c], 0.f),
+                                 fmaxf(__uint_as_float(r1[2 * c + 1]) + sb3[cp * 64 + 33 + 2 * c], 0.f));
+        }
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {   // lane-rotated chunk order: conflict-free 256-B row pitch
+          const int sel = (c + m) & 7;
+          uint4 v = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+#pragma unroll
+          for (int t = 1; t < 8; ++t)
+            if (sel == t) v = make_uint4(pk[4 * t], pk[4 * t + 1], pk[4 * t + 2], pk[4 * t + 3]);
+          *reinterpret_cast<uint4*>(row + (cp * 8 + sel) * 16) = v;
+        }
+      }
+      fence_before();
+      fence_async_smem();                             // staging rows are read by TMA bulk copies
+      __syncwarp();
+      if (lane == 0) { mbar_arrive(c3empty); mbar_arrive(stg_full); }
+      if (q == 0) PSIM_TS(66);
     }
   } else if (warp == cs::WB_WARP) {   // ============================ a4 write-back
-    // copies the 128 staged conv3 rows (256 B each) of a tile to a4[b][p] with
-    // coalesced 256-B stores, off the epilogue's critical path
+    // the 128 staged conv3 rows (256 B each) of a tile -> a4[b][p] by TMA bulk stores,
+    // off the epilogues' critical path
     uint32_t it = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
       uint32_t ids[4];
@@ -350,7 +357,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       }
       wait_full(stg_full, it);
 #pragma unroll
-      for (int u = 0; u < 4; ++u)                   // one 256-B TMA bulk store per row
+      for (int u = 0; u < 4; ++u)
         if (ids[u] != 0xFFFFFFFFu)
           bulk_s2g(a.a4 + ((uint64_t)(ids[u] >> 4) * 14 + (ids[u] & 15)) * 128,
                    sm + cs::A3_OFF + (u * 32 + lane) * 256, 256);
@@ -360,89 +367,108 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (lane == 0) mbar_arrive(stg_empty);
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
-    // Thread (m, h) builds row 2j+h of block m for the 4 conv1 positions j of a
-    // tile.  All loads of a tile are issued up front (block id -> sub-trace state
-    // -> 4 queue entries -> 4 trace rows: 3 dependent round trips per tile
-    // instead of 8), then rows are converted into the A tile as X slots free up.
-    const int g = tid - cs::GATHER_WARP0 * 32;
-    const int m = g & 127, h = g >> 7;
-    uint32_t it = 0;
-    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+    // Thread m builds rows 2j and 2j+1 of block m for the 4 conv1 positions j of
+    // each tile.  Items n = (tile, j) run a 3-stage software pipeline so no
+    // memory latency is exposed: at item n the rows of n are converted into the
+    // A tile, the trace rows of n+1 are loaded (their queue entries arrived) and
+    // the queue entries of n+2 are loaded; block id + sub-trace state of a tile
+    // are loaded two items before its first queue access.
+    const int m = tid - cs::GATHER_WARP0 * 32;
+    struct Meta { uint32_t b; int p, k; uint32_t i, clo; bool valid; };
+    struct Ent { uint32_t row; int t0, t1, t2; bool on; };   // queue part of one input row
+    struct Row { uint4 v0, v1, v2; int t0, t1, t2; bool on; };
+    auto load_meta = [&](uint32_t tl, Meta& mt) {
       const uint32_t bi = tl * cs::TILE + m;
-      const bool valid = bi < nblocks;
-      uint32_t b = 0, p = 0;
-      int k = -1;
-      int64_t i = 0;
-      uint32_t clo = 0;
-      if (valid) {
+      mt.valid = tl < ntiles && bi < nblocks;
+      mt.b = 0; mt.p = 0; mt.k = -1; mt.i = 0; mt.clo = 0;
+      if (mt.valid) {
         const uint32_t id = a.blocks[bi];
-        b = id >> 4; p = id & 15;
-        k = a.count[b];
-        i = a.ws[b] + a.step;
-        clo = (uint32_t)a.clock[b];
+        mt.b = id >> 4; mt.p = (int)(id & 15);
+        mt.k = a.count[mt.b];
+        mt.i = (uint32_t)(a.ws[mt.b] + a.step);
+        mt.clo = (uint32_t)a.clock[mt.b];
       }
-      if (warp == cs::GATHER_WARP0) PSIM_TS(80);
-      int64_t rowj[4];
-      int tf[4][3];
-      bool on[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int R = (int)p * 8 + 2 * j + h;        // input row of this thread
-        on[j] = valid && R <= k;
-        rowj[j] = i;                                 // R == 0: current instruction first
-        tf[j][0] = tf[j][1] = tf[j][2] = 0;
-        if (on[j] && R > 0) {
-          const int e = k - R;                       // context newest first (R6)
-          const uint64_t qo = (uint64_t)e * a.qn + b;
-          rowj[j] = a.q_seq[qo];
-          const uint32_t csv = a.q_cs[qo];
-          const int c = csv & 0xFFFF, sv = csv >> 16;
-          int age = (int)(clo - a.q_fetch[qo]);      // time relative to Clock (R2)
-          int remc = max(0, c - age);
-          int remr = c + sv - age;
-          tf[j][0] = min(age, kTimeMax); tf[j][1] = min(remc, kTimeMax); tf[j][2] = min(remr, kTimeMax);
-        }
+    };
+    auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // queue entry of row 2j+h
+      const int R = mt.p * 8 + 2 * j + h;            // input row (PAPER.md:93 row order)
+      en.on = mt.valid && R <= mt.k;
+      en.t0 = en.t1 = en.t2 = 0;
+      en.row = mt.i;                                 // R == 0: current instruction first
+      if (en.on && R > 0) {
+        const uint64_t qo = (uint64_t)(mt.k - R) * a.qn + mt.b;   // context newest first (R6)
+        en.row = a.q_seq[qo];
+        const uint32_t csv = a.q_cs[qo];
+        const int c = csv & 0xFFFF, sv = csv >> 16;
+        const int age = (int)(mt.clo - a.q_fetch[qo]);   // time relative to Clock (R2)
+        en.t0 = min(age, kTimeMax); en.t1 = min(max(0, c - age), kTimeMax); en.t2 = min(c + sv - age, kTimeMax);
       }
-      uint4 v[4][3];
+    };
+    auto stage_b = [&](const Ent& en, Row& r) {      // the trace row of that entry
+      r.on = en.on; r.t0 = en.t0; r.t1 = en.t1; r.t2 = en.t2;
+      if (en.on) {
+        const uint4* ar = reinterpret_cast<const uint4*>(a.trace + ((int64_t)en.row - a.row_lo) * a.stride);
+        r.v0 = __ldg(ar); r.v1 = __ldg(ar + 1); r.v2 = __ldg(ar + 2);
+      } else {
+        r.v0 = r.v1 = r.v2 = make_uint4(0, 0, 0, 0);
+      }
+    };
+    // 64 bf16 columns of one row: 0..2 time, 3..49 attributes 0..46, 50..63 zero (R1)
+    auto stage_c = [&](const Row& r, uint8_t* atom) {
+      uint32_t w[32];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        if (on[j]) {
-          const uint4* ar = reinterpret_cast<const uint4*>(a.trace + (rowj[j] - a.row_lo) * a.stride);
-          v[j][0] = __ldg(ar); v[j][1] = __ldg(ar + 1); v[j][2] = __ldg(ar + 2);
-        } else {
-          v[j][0] = v[j][1] = v[j][2] = make_uint4(0, 0, 0, 0);
-        }
+      for (int t = 0; t < 32; ++t) w[t] = 0;
+      if (r.on) {
+        const uint32_t by[12] = {r.v0.x, r.v0.y, r.v0.z, r.v0.w, r.v1.x, r.v1.y, r.v1.z, r.v1.w,
+                                 r.v2.x, r.v2.y, r.v2.z, r.v2.w};
+        float f[47];
+#pragma unroll
+        for (int t = 0; t < 47; ++t) f[t] = (float)((by[t >> 2] >> ((t & 3) * 8)) & 0xFFu);
+        w[0] = pack_bf16((float)r.t0, (float)r.t1);
+        w[1] = pack_bf16((float)r.t2, f[0]);
+#pragma unroll
+        for (int t = 2; t < 25; ++t) w[t] = pack_bf16(f[2 * t - 3], f[2 * t - 2]);
       }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int s = j & 1;
-        uint32_t w[32];                              // 64 bf16 values, packed pairs
-#pragma unroll
-        for (int t = 0; t < 32; ++t) w[t] = 0;
-        if (on[j]) {
-          uint32_t by[12];
-          by[0] = v[j][0].x; by[1] = v[j][0].y; by[2] = v[j][0].z; by[3] = v[j][0].w;
-          by[4] = v[j][1].x; by[5] = v[j][1].y; by[6] = v[j][1].z; by[7] = v[j][1].w;
-          by[8] = v[j][2].x; by[9] = v[j][2].y; by[10] = v[j][2].z; by[11] = v[j][2].w;
-#define PSIM_BYTE(idx) ((by[(idx) >> 2] >> (((idx) & 3) * 8)) & 0xFFu)
-          // columns: 0..2 time, 3..49 attributes 0..46, 50..63 zero (R1)
-          w[0] = bf16_bits_int(tf[j][0]) | (bf16_bits_int(tf[j][1]) << 16);
-          w[1] = bf16_bits_int(tf[j][2]) | (bf16_bits_u8(PSIM_BYTE(0)) << 16);
-#pragma unroll
-          for (int t = 2; t < 25; ++t)   // columns 2t, 2t+1 -> attributes 2t-3, 2t-2
-            w[t] = bf16_bits_u8(PSIM_BYTE(2 * t - 3)) | (bf16_bits_u8(PSIM_BYTE(2 * t - 2)) << 16);
-#undef PSIM_BYTE
-        }
-        if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
-        wait_empty(xempty + s, it * 2 + (j >> 1));
-        if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
-        uint8_t* atom = sm + cs::X_OFF + s * 32768 + h * 16384;
-#pragma unroll
-        for (int c = 0; c < 8; ++c) st_sw128(atom, m, c, make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]));
-        fence_async_smem();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(xfull + s);
-        if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
+      for (int c = 0; c < 8; ++c) st_sw128(atom, m, c, make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]));
+    };
+    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const uint32_t n_items = my_tiles * 4;
+    Meta m0, m1, m2;                                  // metas of tiles it, it+1, it+2
+    load_meta(blockIdx.x, m0);
+    load_meta(blockIdx.x + gridDim.x, m1);
+    load_meta(blockIdx.x + 2 * gridDim.x, m2);
+    Ent e1a, e1b, e2a, e2b;                           // queue parts of items n+1, n+2
+    Row r0a, r0b, r1a, r1b;                           // rows of items n, n+1
+    if (n_items > 0) {
+      stage_a(m0, 0, 0, e1a); stage_a(m0, 0, 1, e1b);
+      stage_b(e1a, r0a); stage_b(e1b, r0b);           // item 0: rows
+      stage_a(m0, 1, 0, e1a); stage_a(m0, 1, 1, e1b); // item 1: queue entries
+    }
+#pragma unroll 1
+    for (uint32_t nI = 0; nI < n_items; ++nI) {
+      const uint32_t it = nI >> 2;
+      const int j = (int)(nI & 3), s = j & 1;
+      if (nI + 1 < n_items) { stage_b(e1a, r1a); stage_b(e1b, r1b); }          // rows of n+1
+      if (nI + 2 < n_items) {                                                  // entries of n+2
+        const int j2 = (int)((nI + 2) & 3);
+        const Meta& mm = j2 >= 2 ? m0 : m1;      // n+2 is in tile it (j <= 1) or it+1 (j >= 2)
+        stage_a(mm, j2, 0, e2a); stage_a(mm, j2, 1, e2b);
+      }
+      if (j == 0 && warp == cs::GATHER_WARP0) PSIM_TS(80);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      wait_empty(xempty + s, it * 2 + (j >> 1));
+      if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
+      stage_c(r0a, sm + cs::X_OFF + s * 32768);
+      stage_c(r0b, sm + cs::X_OFF + s * 32768 + 16384);
+      fence_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(xfull + s);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
+      r0a = r1a; r0b = r1b;
+      e1a = e2a; e1b = e2b;
+      if (j == 3) {                                   // next tile: rotate metas, load tile it+3's
+        m0 = m1; m1 = m2;
+        load_meta(blockIdx.x + (it + 3) * gridDim.x, m2);
       }
     }
   }
