@@ -55,8 +55,8 @@ struct ConvArgs {
   const uint32_t* blocks;    // block ids (b << 4 | p) of this step
   const uint32_t* nblocks;   // count of this step's list
   uint32_t* next_count;      // the other step parity's counter, reset here
-  const uint8_t* trace;
-  int64_t row_lo, stride;
+  const __nv_bfloat16* trace16;   // [rows][64] bf16 operand rows (attributes at cols 0..46)
+  int64_t row_lo;
   const int64_t* ws;
   const int64_t* clock;
   const int32_t* count;
@@ -368,108 +368,104 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
     // Thread m builds rows 2j and 2j+1 of block m for the 4 conv1 positions j of
-    // each tile.  Items n = (tile, j) run a 3-stage software pipeline so no
-    // memory latency is exposed: at item n the rows of n are converted into the
-    // A tile, the trace rows of n+1 are loaded (their queue entries arrived) and
-    // the queue entries of n+2 are loaded; block id + sub-trace state of a tile
-    // are loaded two items before its first queue access.
+    // each tile.  Operand row layout (per input row, 64 bf16): cols 0..46 the
+    // trace attributes (pre-converted once per run into trace16, copied with
+    // cp.async straight into the SWIZZLE_128B tile), col 47 zero, cols 48..50 the
+    // time features (one 16-byte store), cols 51..63 zero (chunk 7 is zeroed
+    // once).  The copies of item n are in flight while item n-1 is signalled:
+    // xfull(n-1) is arrived after cp.async.wait_group<1> + fence.proxy.async.
+    // No load result is consumed in the iteration that issues it: block ids of
+    // tile t+2 are loaded at position 0 of tile t, their sub-trace state at
+    // position 2, queue entries of item n+1 during item n.
     const int m = tid - cs::GATHER_WARP0 * 32;
     struct Meta { uint32_t b; int p, k; uint32_t i, clo; bool valid; };
-    struct Ent { uint32_t row; int t0, t1, t2; bool on; };   // queue part of one input row
-    struct Row { uint4 v0, v1, v2; int t0, t1, t2; bool on; };
-    auto load_meta = [&](uint32_t tl, Meta& mt) {
+    struct Ent { uint32_t seq, fet, csv; int kind; };   // kind: 0 padding, 1 current, 2 context
+    auto meta_ids = [&](uint32_t tl, Meta& mt) {         // stage 1: block id
       const uint32_t bi = tl * cs::TILE + m;
       mt.valid = tl < ntiles && bi < nblocks;
-      mt.b = 0; mt.p = 0; mt.k = -1; mt.i = 0; mt.clo = 0;
+      mt.b = mt.valid ? a.blocks[bi] : 0u;               // raw id until meta_state
+    };
+    auto meta_state = [&](Meta& mt) {                    // stage 2: sub-trace state
+      const uint32_t id = mt.b;
+      mt.b = id >> 4; mt.p = (int)(id & 15);
+      mt.k = -1; mt.i = 0; mt.clo = 0;
       if (mt.valid) {
-        const uint32_t id = a.blocks[bi];
-        mt.b = id >> 4; mt.p = (int)(id & 15);
         mt.k = a.count[mt.b];
         mt.i = (uint32_t)(a.ws[mt.b] + a.step);
         mt.clo = (uint32_t)a.clock[mt.b];
       }
     };
-    auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // queue entry of row 2j+h
+    auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // raw queue entry of row 2j+h
       const int R = mt.p * 8 + 2 * j + h;            // input row (PAPER.md:93 row order)
-      en.on = mt.valid && R <= mt.k;
-      en.t0 = en.t1 = en.t2 = 0;
-      en.row = mt.i;                                 // R == 0: current instruction first
-      if (en.on && R > 0) {
+      en.kind = (mt.valid && R <= mt.k) ? (R == 0 ? 1 : 2) : 0;
+      en.seq = mt.i; en.fet = 0; en.csv = 0;         // R == 0: current instruction first
+      if (en.kind == 2) {
         const uint64_t qo = (uint64_t)(mt.k - R) * a.qn + mt.b;   // context newest first (R6)
-        en.row = a.q_seq[qo];
-        const uint32_t csv = a.q_cs[qo];
-        const int c = csv & 0xFFFF, sv = csv >> 16;
-        const int age = (int)(mt.clo - a.q_fetch[qo]);   // time relative to Clock (R2)
-        en.t0 = min(age, kTimeMax); en.t1 = min(max(0, c - age), kTimeMax); en.t2 = min(c + sv - age, kTimeMax);
+        en.seq = a.q_seq[qo]; en.fet = a.q_fetch[qo]; en.csv = a.q_cs[qo];
       }
     };
-    auto stage_b = [&](const Ent& en, Row& r) {      // the trace row of that entry
-      r.on = en.on; r.t0 = en.t0; r.t1 = en.t1; r.t2 = en.t2;
-      if (en.on) {
-        const uint4* ar = reinterpret_cast<const uint4*>(a.trace + ((int64_t)en.row - a.row_lo) * a.stride);
-        r.v0 = __ldg(ar); r.v1 = __ldg(ar + 1); r.v2 = __ldg(ar + 2);
+    auto issue = [&](const Ent& en, uint32_t clo, uint8_t* atom) {   // one input row -> row m of an X atom
+      if (en.kind) {
+        int t0 = 0, t1 = 0, t2 = 0;
+        if (en.kind == 2) {                          // time relative to Clock (R2)
+          const int c = en.csv & 0xFFFF, sv = en.csv >> 16;
+          const int age = (int)(clo - en.fet);
+          t0 = min(age, kTimeMax); t1 = min(max(0, c - age), kTimeMax); t2 = min(c + sv - age, kTimeMax);
+        }
+        const uint8_t* src = reinterpret_cast<const uint8_t*>(a.trace16 + ((int64_t)en.seq - a.row_lo) * 64);
+#pragma unroll
+        for (int c = 0; c < 6; ++c) cp_async16(atom + m * 128 + ((c ^ (m & 7)) << 4), src + c * 16);
+        st_sw128(atom, m, 6, make_uint4(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f), 0u, 0u));
       } else {
-        r.v0 = r.v1 = r.v2 = make_uint4(0, 0, 0, 0);
+#pragma unroll
+        for (int c = 0; c < 7; ++c) st_sw128(atom, m, c, make_uint4(0, 0, 0, 0));
       }
     };
-    // 64 bf16 columns of one row: 0..2 time, 3..49 attributes 0..46, 50..63 zero (R1)
-    auto stage_c = [&](const Row& r, uint8_t* atom) {
-      uint32_t w[32];
+    // chunk 7 (cols 56..63) of every X row is always zero
 #pragma unroll
-      for (int t = 0; t < 32; ++t) w[t] = 0;
-      if (r.on) {
-        const uint32_t by[12] = {r.v0.x, r.v0.y, r.v0.z, r.v0.w, r.v1.x, r.v1.y, r.v1.z, r.v1.w,
-                                 r.v2.x, r.v2.y, r.v2.z, r.v2.w};
-        float f[47];
+    for (int s2 = 0; s2 < 2; ++s2)
 #pragma unroll
-        for (int t = 0; t < 47; ++t) f[t] = (float)((by[t >> 2] >> ((t & 3) * 8)) & 0xFFu);
-        w[0] = pack_bf16((float)r.t0, (float)r.t1);
-        w[1] = pack_bf16((float)r.t2, f[0]);
-#pragma unroll
-        for (int t = 2; t < 25; ++t) w[t] = pack_bf16(f[2 * t - 3], f[2 * t - 2]);
-      }
-#pragma unroll
-      for (int c = 0; c < 8; ++c) st_sw128(atom, m, c, make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]));
-    };
+      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const uint32_t n_items = my_tiles * 4;
-    Meta m0, m1, m2;                                  // metas of tiles it, it+1, it+2
-    load_meta(blockIdx.x, m0);
-    load_meta(blockIdx.x + gridDim.x, m1);
-    load_meta(blockIdx.x + 2 * gridDim.x, m2);
-    Ent e1a, e1b, e2a, e2b;                           // queue parts of items n+1, n+2
-    Row r0a, r0b, r1a, r1b;                           // rows of items n, n+1
-    if (n_items > 0) {
-      stage_a(m0, 0, 0, e1a); stage_a(m0, 0, 1, e1b);
-      stage_b(e1a, r0a); stage_b(e1b, r0b);           // item 0: rows
-      stage_a(m0, 1, 0, e1a); stage_a(m0, 1, 1, e1b); // item 1: queue entries
-    }
+    Meta m0, m1, m2;                                  // tiles it, it+1, it+2
+    meta_ids(blockIdx.x, m0);
+    meta_ids(blockIdx.x + gridDim.x, m1);
+    meta_state(m0);
+    meta_state(m1);
+    Ent ea, eb;                                       // raw queue parts of item n
+    if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
       const int j = (int)(nI & 3), s = j & 1;
-      if (nI + 1 < n_items) { stage_b(e1a, r1a); stage_b(e1b, r1b); }          // rows of n+1
-      if (nI + 2 < n_items) {                                                  // entries of n+2
-        const int j2 = (int)((nI + 2) & 3);
-        const Meta& mm = j2 >= 2 ? m0 : m1;      // n+2 is in tile it (j <= 1) or it+1 (j >= 2)
-        stage_a(mm, j2, 0, e2a); stage_a(mm, j2, 1, e2b);
-      }
+      if (j == 0) meta_ids(blockIdx.x + (it + 2) * gridDim.x, m2);
+      if (j == 2) meta_state(m2);
       if (j == 0 && warp == cs::GATHER_WARP0) PSIM_TS(80);
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
       wait_empty(xempty + s, it * 2 + (j >> 1));
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
-      stage_c(r0a, sm + cs::X_OFF + s * 32768);
-      stage_c(r0b, sm + cs::X_OFF + s * 32768 + 16384);
+      issue(ea, m0.clo, sm + cs::X_OFF + s * 32768);
+      issue(eb, m0.clo, sm + cs::X_OFF + s * 32768 + 16384);
+      cp_async_commit();
+      if (nI + 1 < n_items) {                         // raw queue entries of item n+1
+        const Meta& mm = j == 3 ? m1 : m0;
+        stage_a(mm, (j + 1) & 3, 0, ea); stage_a(mm, (j + 1) & 3, 1, eb);
+      }
+      if (nI > 0) {                                   // item n-1 landed -> visible to tcgen05
+        cp_async_wait<1>();
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(xfull + ((j + 1) & 1));
+      }
+      if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
+      if (j == 3) { m0 = m1; m1 = m2; }               // next tile
+    }
+    if (n_items > 0) {                                // the last item
+      cp_async_wait<0>();
       fence_async_smem();
       __syncwarp();
-      if (lane == 0) mbar_arrive(xfull + s);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
-      r0a = r1a; r0b = r1b;
-      e1a = e2a; e1b = e2b;
-      if (j == 3) {                                   // next tile: rotate metas, load tile it+3's
-        m0 = m1; m1 = m2;
-        load_meta(blockIdx.x + (it + 3) * gridDim.x, m2);
-      }
+      if (lane == 0) mbar_arrive(xfull + (((n_items - 1) & 3) & 1));
     }
   }
   fence_before();
@@ -732,6 +728,30 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   }
 }
 
+// trace rows -> bf16 operand rows: cols 0..46 = attributes (exact: integers < 256),
+// cols 47..63 = 0 (time features are inserted by the gather at cols 48..50)
+__global__ void trace16_kernel(const uint8_t* __restrict__ trace, int64_t stride, int64_t rows,
+                               __nv_bfloat16* __restrict__ out) {
+  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;   // one 16-B output chunk
+  if (t >= rows * 8) return;
+  const int64_t r = t >> 3;
+  const int c = (int)(t & 7);
+  const uint8_t* src = trace + r * stride;
+  uint32_t w[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const int a0 = c * 8 + 2 * q, a1 = a0 + 1;
+    const float f0 = a0 < 47 ? (float)src[a0] : 0.f;
+    const float f1 = a1 < 47 ? (float)src[a1] : 0.f;
+    w[q] = pack_bf16(f0, f1);
+  }
+  reinterpret_cast<uint4*>(out)[t] = make_uint4(w[0], w[1], w[2], w[3]);
+}
+void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st) {
+  const int64_t n = rows * 8;
+  if (n > 0) trace16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(trace, stride, rows, out);
+}
+
 // step-0 block list: every sub-trace has k = 0 -> P = 1
 __global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count, uint8_t* tileP, uint32_t* next_count) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -819,7 +839,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   a.blocks = f.blocks;
   a.nblocks = f.count + (step & 1);
   a.next_count = f.count + ((step + 1) & 1);
-  a.trace = g.trace; a.row_lo = g.row_lo; a.stride = g.stride;
+  a.trace16 = f.trace16; a.row_lo = g.row_lo;
   a.ws = g.ws; a.clock = g.clock; a.count = g.count;
   a.q_seq = g.q_seq; a.q_fetch = g.q_fetch; a.q_cs = g.q_cs;
   a.step = step;
@@ -860,7 +880,7 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
 }
 
 bool fused_make_weight_maps(FusedC3& f) {
-  return map2d(&f.mapW1, f.w1, 64, 128, 64) && map2d(&f.mapW2, f.w2, 128, 128, 128) &&
+  return map2d(&f.mapW1, f.w1p, 64, 128, 64) && map2d(&f.mapW2, f.w2, 128, 128, 128) &&
          map2d(&f.mapW3, f.w3, 128, 256, 128);
 }
 

@@ -135,6 +135,10 @@ struct FusedC3 {
   const __nv_bfloat16* wfc1 = nullptr;
   const float *b1 = nullptr, *b2 = nullptr, *b3 = nullptr;
   float* T = nullptr;                 // [15][256] constant fc1 table (owned)
+  __nv_bfloat16* w1p = nullptr;       // conv1 weight [64][128] in the fused row layout (owned):
+                                      // per tap h: cols 0..46 attributes, 48..50 time features
+  __nv_bfloat16* trace16 = nullptr;   // per-run bf16 copy of the rank's trace rows [rows][64] (owned)
+  size_t trace16_cap = 0;
   const float* head_w = nullptr;      // fc2 [3][256]
   const float* head_b = nullptr;
   // per-run buffers (owned), sized for cap_n sub-traces
@@ -147,6 +151,8 @@ struct FusedC3 {
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
 };
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
+// trace rows (uint8 attributes) -> bf16 operand rows of the fused conv1 layout
+void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st);
 void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n, cudaStream_t st);
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
                      cudaStream_t st);

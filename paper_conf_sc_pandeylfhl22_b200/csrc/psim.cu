@@ -220,6 +220,8 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->rec_k);
   dfree(ctx->rec_clock);
   dfree(ctx->fused.T);
+  dfree(ctx->fused.w1p);
+  dfree(ctx->fused.trace16);
   dfree(ctx->fused.blocks);
   dfree(ctx->fused.count);
   dfree(ctx->fused.tileP[0]);
@@ -413,7 +415,6 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
     const float* W2 = B1 + 64;        const float* B2 = W2 + 128 * 64 * 2;
     const float* W3 = B2 + 128;       const float* B3 = W3 + 128 * 128 * 2;
     const float* WF = B3 + 128;       const float* BF = WF + 256 * 1792;
-    (void)W1;
     double r1[64], r2[128], c3[128];
     for (int o = 0; o < 64; ++o) r1[o] = bf(std::max(0.0, (double)B1[o]));
     for (int o = 0; o < 128; ++o) {
@@ -438,6 +439,17 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
     CK(cudaMalloc(&fz.T, T.size() * 4));
     CK(cudaMemcpy(fz.T, T.data(), T.size() * 4, cudaMemcpyHostToDevice));
     fz.w1 = (const __nv_bfloat16*)m.layers[0].w; fz.b1 = m.layers[0].bias;
+    {   // conv1 weight in the fused row layout: K = h*64 + col, col < 47 attribute col-3.., 48..50 time
+      std::vector<uint16_t> w1p((size_t)64 * 128, 0);
+      for (int o = 0; o < 64; ++o)
+        for (int h = 0; h < 2; ++h) {
+          for (int a = 0; a < 47; ++a) w1p[(size_t)o * 128 + h * 64 + a] = f32_to_bf16_rne(W1[((size_t)o * 50 + 3 + a) * 2 + h]);
+          for (int t = 0; t < 3; ++t) w1p[(size_t)o * 128 + h * 64 + 48 + t] = f32_to_bf16_rne(W1[((size_t)o * 50 + t) * 2 + h]);
+        }
+      dfree(fz.w1p);
+      CK(cudaMalloc(&fz.w1p, w1p.size() * 2));
+      CK(cudaMemcpy(fz.w1p, w1p.data(), w1p.size() * 2, cudaMemcpyHostToDevice));
+    }
     fz.w2 = (const __nv_bfloat16*)m.layers[1].w; fz.b2 = m.layers[1].bias;
     fz.w3 = (const __nv_bfloat16*)m.layers[2].w; fz.b3 = m.layers[2].bias;
     fz.wfc1 = (const __nv_bfloat16*)m.layers[3].w;
@@ -581,7 +593,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
 
   int rc = ensure_state(ctx);
   if (rc) return rc;
-  const bool fused = predict && ctx->fused.ready && !(ctx->opts.flags & PSIM_LAYERWISE) && (ctx->stride % 16) == 0;
+  const bool fused = predict && ctx->fused.ready && !(ctx->opts.flags & PSIM_LAYERWISE);
   if (predict && !fused) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
   if (fused) {
     FusedC3& fz = ctx->fused;
@@ -648,6 +660,17 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
   if (fused && n) {
+    // bf16 operand rows of the rank's trace (once per run; the trace crosses HBM once more)
+    const size_t t16 = (size_t)rows * 128;
+    if (ctx->fused.trace16_cap < t16) {
+      dfree(ctx->fused.trace16);
+      ctx->fused.trace16 = nullptr;
+      CK(cudaMalloc(&ctx->fused.trace16, t16 + 256));
+      ctx->fused.trace16_cap = t16;
+    }
+    pf.begin(PSIM_KC_OTHER);
+    launch_trace16(dtr, (int64_t)ctx->stride, rows, ctx->fused.trace16, st);
+    pf.end(PSIM_KC_OTHER);
     // invariant of the fused path: a4 rows p >= P_b are zero (fc1 reads them as 0)
     CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
     pf.begin(PSIM_KC_OTHER);

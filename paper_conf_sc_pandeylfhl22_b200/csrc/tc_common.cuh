@@ -60,6 +60,13 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 // wait until this thread's bulk copies have finished READING their smem source
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+// Ampere-style 16-byte async copy global -> shared (L2 only), grouped
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 // K-major SWIZZLE_128B shared-memory matrix descriptor: LBO 16 B (unused for
 // swizzled K-major), SBO 1024 B between 8-row core-matrix groups, version 1,
 // layout type 2 (SWIZZLE_128B).  The tile base must be 1024-byte aligned.
