@@ -273,7 +273,7 @@ def main():
         return float(t.item())
 
     sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=rank, world_size=world, nccl_id=nccl_id,
-                      stream=stream.cuda_stream, profile=True)
+                      stream=stream.cuda_stream, profile=True, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")))
     sim.load_model(cfg["arch"], w)
 
     def timed(trace_tensor, k_steps, warm):

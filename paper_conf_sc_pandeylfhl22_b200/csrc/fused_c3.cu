@@ -752,6 +752,55 @@ void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfl
   if (n > 0) trace16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(trace, stride, rows, out);
 }
 
+// one warp per sub-trace: rows [ws + t0, min(e, ws + t1)) of a pinned, device-mapped
+// host trace (48-byte rows, contiguous per sub-trace) -> bf16 operand rows.  Lane l
+// reads 16-byte segment q = l % 3 of row l / 3 (10 rows, 480 contiguous bytes per
+// warp step, 4 steps in flight) and writes output chunks 2q, 2q+1 (+ the zero chunks
+// 6, 7 for q = 2).  No shared memory, 128 threads: co-resides with the persistent
+// compute kernels, so the copy overlaps the simulation.
+__global__ void __launch_bounds__(128) load_chunk16_kernel(const uint8_t* __restrict__ host, int64_t host_first_row,
+                                                           int64_t stride, const int64_t* __restrict__ ws,
+                                                           const int64_t* __restrict__ e, uint64_t n, int64_t t0,
+                                                           int64_t t1, int64_t row_lo, __nv_bfloat16* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
+  const int rl = lane / 3, q = lane % 3;
+  for (uint64_t b = warp; b < n; b += nwarps) {
+    const int64_t r0 = ws[b] + t0;
+    const int64_t r1 = min(e[b], ws[b] + t1);
+#pragma unroll 4
+    for (int64_t rb = r0; rb < r1; rb += 10) {
+      const int64_t r = rb + rl;
+      if (lane < 30 && r < r1) {
+        const uint4 v = *reinterpret_cast<const uint4*>(host + (r - host_first_row) * stride + q * 16);
+        const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+        uint32_t o[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          const int a0 = q * 16 + 2 * t, a1 = a0 + 1;   // attribute indices (cols 0..46 of the output row)
+          const float f0 = a0 < 47 ? (float)((wv[(2 * t) >> 2] >> (((2 * t) & 3) * 8)) & 0xFFu) : 0.f;
+          const float f1 = a1 < 47 ? (float)((wv[(2 * t + 1) >> 2] >> (((2 * t + 1) & 3) * 8)) & 0xFFu) : 0.f;
+          o[t] = pack_bf16(f0, f1);
+        }
+        uint4* dst = reinterpret_cast<uint4*>(out + (r - row_lo) * 64);
+        dst[2 * q] = make_uint4(o[0], o[1], o[2], o[3]);
+        dst[2 * q + 1] = make_uint4(o[4], o[5], o[6], o[7]);
+        if (q == 2) { dst[6] = make_uint4(0, 0, 0, 0); dst[7] = make_uint4(0, 0, 0, 0); }
+      }
+    }
+  }
+}
+void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64_t stride, const int64_t* ws,
+                         const int64_t* e, uint64_t n, int64_t t0, int64_t t1, int64_t row_lo,
+                         __nv_bfloat16* trace16, cudaStream_t st) {
+  uint64_t blocks = (n * 32 + 127) / 128;
+  if (blocks > 148ull * 2) blocks = 148ull * 2;   // ~one 4-warp CTA per SM next to the compute kernels
+  if (blocks < 1) blocks = 1;
+  load_chunk16_kernel<<<(unsigned)blocks, 128, 0, st>>>(host_rows, host_first_row, stride, ws, e, n, t0, t1, row_lo,
+                                                         trace16);
+}
+
 // step-0 block list: every sub-trace has k = 0 -> P = 1
 __global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count, uint8_t* tileP, uint32_t* next_count) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;

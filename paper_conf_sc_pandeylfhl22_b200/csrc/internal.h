@@ -153,6 +153,11 @@ struct FusedC3 {
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
 // trace rows (uint8 attributes) -> bf16 operand rows of the fused conv1 layout
 void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st);
+// streamed variant for pinned host traces: the rows sub-trace b touches in lockstep
+// steps [t0, t1) are read over PCIe (zero-copy) and written as bf16 operand rows
+void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64_t stride, const int64_t* ws,
+                         const int64_t* e, uint64_t n, int64_t t0, int64_t t1, int64_t row_lo,
+                         __nv_bfloat16* trace16, cudaStream_t st);
 void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n, cudaStream_t st);
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
                      cudaStream_t st);

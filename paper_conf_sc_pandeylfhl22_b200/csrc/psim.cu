@@ -114,6 +114,9 @@ struct psim_ctx {
   int trace_mode = 0;
   uint8_t* d_trace = nullptr;
   size_t d_trace_cap = 0;
+  const uint8_t* trace_devptr = nullptr;   // device-accessible address of a pinned host trace
+  cudaStream_t ld_stream = nullptr;        // trace streaming (pinned host traces, fused path)
+  std::vector<cudaEvent_t> ld_events;
   // partition
   bool partitioned = false;
   uint64_t N = 0, W = 0, j0 = 0, j1 = 0;
@@ -204,6 +207,8 @@ void psim_destroy(psim_ctx* ctx) {
   if (ctx->comm && g_nccl.ok) g_nccl.commDestroy(ctx->comm);
   dfree(ctx->d_trace);
   dfree(ctx->d_forced);
+  for (auto e : ctx->ld_events) cudaEventDestroy(e);
+  if (ctx->ld_stream) cudaStreamDestroy(ctx->ld_stream);
   for (auto& l : ctx->model.layers) { dfree(l.w); dfree(l.bias); }
   dfree(ctx->model.head_w);
   dfree(ctx->model.head_b);
@@ -253,6 +258,14 @@ int psim_load_trace(psim_ctx* ctx, const uint8_t* attrs, uint64_t n_instr, uint6
   }
   cudaGetLastError();
   if (mode == 0 && (row_stride % 16)) FAIL(PSIM_ERR_ARG, "device trace row_stride must be a multiple of 16");
+  ctx->trace_devptr = nullptr;
+  if (mode == 1) {
+    void* dp = nullptr;
+    if (cudaHostGetDevicePointer(&dp, const_cast<uint8_t*>(attrs), 0) == cudaSuccess && dp &&
+        (row_stride % 16) == 0 && (reinterpret_cast<uintptr_t>(dp) % 16) == 0)
+      ctx->trace_devptr = static_cast<const uint8_t*>(dp);
+    cudaGetLastError();
+  }
   if (ctx->L != n_instr) ctx->partitioned = false;
   ctx->trace = attrs;
   ctx->L = n_instr;
@@ -631,8 +644,14 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
 
   // ---- trace: the rank's rows cross the host link once ----
   CK(cudaEventRecord(ctx->ev[0], st));
-  const uint8_t* dtr;
-  if (ctx->trace_mode == 0) {
+  // pinned host trace + fused path: stream it in chunks of lockstep steps, overlapped with
+  // the simulation (the paper's pipelined copy, :163), converting to bf16 operand rows on the way
+  const bool stream_load = fused && n && ctx->trace_mode == 1 && ctx->trace_devptr;
+  const int64_t chunk = ctx->opts.chunk_steps ? (int64_t)ctx->opts.chunk_steps : 64;
+  const uint8_t* dtr = nullptr;
+  if (stream_load) {
+    stats.h2d_bytes = (size_t)rows * 48;
+  } else if (ctx->trace_mode == 0) {
     dtr = ctx->trace + (ctx->row_lo - (int64_t)ctx->first_row) * ctx->stride;
   } else {
     const size_t bytes = (size_t)rows * ctx->stride;
@@ -668,9 +687,27 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       CK(cudaMalloc(&ctx->fused.trace16, t16 + 256));
       ctx->fused.trace16_cap = t16;
     }
-    pf.begin(PSIM_KC_OTHER);
-    launch_trace16(dtr, (int64_t)ctx->stride, rows, ctx->fused.trace16, st);
-    pf.end(PSIM_KC_OTHER);
+    if (stream_load) {
+      if (!ctx->ld_stream) CK(cudaStreamCreateWithFlags(&ctx->ld_stream, cudaStreamNonBlocking));
+      const size_t nch = (size_t)((ctx->steps + chunk - 1) / chunk);
+      while (ctx->ld_events.size() < nch) {
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        ctx->ld_events.push_back(e);
+      }
+      CK(cudaStreamWaitEvent(ctx->ld_stream, ctx->ev[0], 0));
+      for (size_t c = 0; c < nch; ++c) {
+        launch_load_chunk16(ctx->trace_devptr, (int64_t)ctx->first_row, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e,
+                            n, (int64_t)c * chunk, (int64_t)(c + 1) * chunk, ctx->row_lo, ctx->fused.trace16,
+                            ctx->ld_stream);
+        CK(cudaEventRecord(ctx->ld_events[c], ctx->ld_stream));
+      }
+      pf.launches[PSIM_KC_OTHER] += nch;
+    } else {
+      pf.begin(PSIM_KC_OTHER);
+      launch_trace16(dtr, (int64_t)ctx->stride, rows, ctx->fused.trace16, st);
+      pf.end(PSIM_KC_OTHER);
+    }
     // invariant of the fused path: a4 rows p >= P_b are zero (fc1 reads them as 0)
     CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
     pf.begin(PSIM_KC_OTHER);
@@ -678,6 +715,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     pf.end(PSIM_KC_OTHER);
   }
   for (int64_t t = 0; t < ctx->steps && n; ++t) {
+    if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
     if (fused) {
       ga.step = t;
       ua.step = t;

@@ -322,3 +322,32 @@ def test_s3_config3_full_size_sampled():
     assert decision_parity(tr, N, "C3", w, "bf16", samples=[0, 40000, 65535]) >= 0.999
     rel, agree, g = free_running(tr, N, 110, "C3", w, "bf16", samples=[0, 1, 9999, 32768, 40000, 65535])
     assert rel <= 0.005, (rel, agree)
+
+
+@pytest.mark.parametrize("chunk", [0, 7])
+def test_trace_residency_modes_identical(chunk):
+    """The fused path gives bit-identical results whether the trace is resident in HBM,
+    streamed from pinned host memory in chunks of lockstep steps (overlapped with the
+    simulation), or staged from pageable memory."""
+    L, N, W = 20_000, 64, 100
+    tr = synth.trace(L, 4321)
+    w = synth.weights("C3")
+    totals, cycles = [], []
+    pinned = torch.from_numpy(tr).pin_memory()
+    for mode in ("device", "pinned", "pageable"):
+        with P.Simulator(precision="bf16", chunk_steps=chunk) as sim:
+            if mode == "device":
+                sim.load_trace(torch.from_numpy(tr).cuda())
+            elif mode == "pinned":
+                sim.load_trace(pinned)
+            else:
+                sim.load_trace(tr)
+            sim.partition(N, W)
+            sim.load_model("C3", w)
+            sim.simulate()
+            totals.append(sim.total_cycles())
+            cycles.append(sim.subtrace_cycles())
+            st = sim.stats()
+            assert st["trace_mode"] == {"device": 0, "pinned": 1, "pageable": 2}[mode]
+    assert totals[0] == totals[1] == totals[2]
+    assert np.array_equal(cycles[0], cycles[1]) and np.array_equal(cycles[0], cycles[2])
