@@ -74,6 +74,13 @@ def lib():
             P, c.c_long, c.c_long, c.c_long, c.c_long, c.c_int,  # trace, stride, L, N, W, cap
             P, c.c_long, c.c_long, c.c_int64,   # forced, j0, nj, clock0
             P, P, P, P, P, P, P]                # cycles, boundary, lat, y, k, clock, stalls
+        _lib.oracle_simulate_pec.restype = c.c_int
+        _lib.oracle_simulate_pec.argtypes = [
+            c.c_int, c.c_int, P, c.c_long,      # arch, mode, weights, n
+            P, c.c_long, c.c_long, c.c_long, c.c_long, c.c_int,  # trace, stride, L, N, W, cap
+            P, c.c_long, c.c_long, c.c_long, c.c_long,   # forced, j0, nj, G, limit
+            P, P, P, P,                         # cycles, cycles1, boundary, corr_len
+            P, P, P, P, P, P]                   # lat, k, clock, corr_lat, corr_k, stalls
     return _lib
 
 
@@ -184,4 +191,47 @@ def simulate(trace: np.ndarray, N: int, W: int, *, arch: str = "C3", weights=Non
                stalls=int(stalls.value))
     if want_rows:
         out.update(lat=lat, y=y, k=k, clock=clk)
+    return out
+
+
+def simulate_pec(trace: np.ndarray, N: int, W: int, *, limit: int = 100, G: int = 1, arch: str = "C3",
+                 weights=None, mode: int = FP64, cap: int = 110, forced_lat=None, j0: int = 0, nj=None,
+                 want_rows: bool = True, L: int | None = None, row_offset: int = 0):
+    """Simulate with post-error correction (Fig. 9; R19).
+
+    Same arguments as simulate() plus ``limit`` (max re-simulated rows per
+    sub-trace, PAPER.md:291 uses 100) and ``G`` (ranks: the first sub-trace of
+    each rank is not corrected).  Returns dict(cycles (corrected), cycles1
+    (first pass), boundary, corr_len, total, total1, stalls, and per-row
+    lat/k/clock (first pass) and corr_lat/corr_k (re-simulated rows, k = -1
+    elsewhere) over all L rows if want_rows).
+    """
+    trace = np.ascontiguousarray(trace, dtype=np.uint8)
+    L = trace.shape[0] + row_offset if L is None else L
+    nj = N - j0 if nj is None else nj
+    w = None if weights is None else np.ascontiguousarray(weights, dtype=np.float32)
+    forced = None if forced_lat is None else np.ascontiguousarray(forced_lat, dtype=np.uint16)
+    m = max(nj, 1)
+    cycles, cycles1, boundary = (np.zeros(m, np.int64) for _ in range(3))
+    corr_len = np.zeros(m, np.int32)
+    lat = k = clk = clat = ck = None
+    if want_rows:
+        lat = np.zeros((L, 3), np.uint16)
+        k = np.full(L, -1, np.int32)
+        clk = np.zeros(L, np.int64)
+        clat = np.zeros((L, 3), np.uint16)
+        ck = np.full(L, -1, np.int32)
+    stalls = ctypes.c_int64(0)
+    rc = lib().oracle_simulate_pec(
+        ARCH.get(arch, 0), mode, _ptr(w), 0 if w is None else w.size,
+        ctypes.c_void_p(trace.ctypes.data - row_offset * trace.shape[1]), trace.shape[1], L, N, W, cap,
+        _ptr(forced), j0, nj, G, limit,
+        _ptr(cycles), _ptr(cycles1), _ptr(boundary), _ptr(corr_len),
+        _ptr(lat), _ptr(k), _ptr(clk), _ptr(clat), _ptr(ck), ctypes.byref(stalls))
+    if rc != 0:
+        raise ValueError(f"oracle_simulate_pec rc={rc}")
+    out = dict(cycles=cycles[:nj], cycles1=cycles1[:nj], boundary=boundary[:nj], corr_len=corr_len[:nj],
+               total=int(cycles[:nj].sum()), total1=int(cycles1[:nj].sum()), stalls=int(stalls.value))
+    if want_rows:
+        out.update(lat=lat, k=k, clock=clk, corr_lat=clat, corr_k=ck)
     return out

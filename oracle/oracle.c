@@ -400,3 +400,129 @@ int oracle_simulate(int arch, int mode, const float* weights, long n_weights,
     free(We);
     return 0;
 }
+
+/* ------------------------------------------------------------------ */
+/* Post-error correction (PAPER.md:203-219 [V-B "Post-error           */
+/* correction"], Fig. 9; limit :291; R19).                   */
+/*                                                                     */
+/* First pass: every sub-trace j in [j0, j0+nj) exactly as             */
+/* oracle_simulate (warm-up is still used, :205).  Then "if this        */
+/* partition is not the last one on the GPU, it will re-simulate the    */
+/* following instructions, which were previously simulated by the next  */
+/* partition" (:207): sub-trace j's final queue and Clock continue over */
+/* rows i = s_{j+1}, s_{j+1}+1, ...  Before row i is re-simulated the    */
+/* re-simulation's context count is compared with the count the first  */
+/* pass of j+1 saw at row i; the re-simulation "continues until either  */
+/* the number of context instructions of the re-simulation matches the */
+/* prior outcomes or a user-defined resimulation limit" (:219): the     */
+/* first matching row is not re-simulated (Fig. 9: partition 0          */
+/* re-simulates {I4, I5}, terminating at I6), at most `limit` rows are  */
+/* re-simulated, and never past e_{j+1}.  "The re-simulated cycles will */
+/* replace the previously simulated ones" (:207):                       */
+/*   cycles_{j+1} += (Clock_re,last - Clock_{j,end})                    */
+/*                 - (Clock1_{j+1}(last re-simulated row) - bnd_{j+1}).  */
+/* "We do not perform post-error correction for the first partition of */
+/* each GPU" (:219): with G ranks (rank g owns [floor(gN/G),             */
+/* floor((g+1)N/G))), j+1 is corrected only if j is on the same rank;   */
+/* j+1 == j0 (j outside the simulated range) is not corrected either.   */
+/* Sub-traces are processed in index order with j's first-pass final    */
+/* state kept until j+1 has been corrected; the passes are independent  */
+/* so this equals running all first passes before all corrections.      */
+/*                                                                     */
+/* Outputs as oracle_simulate (cycles are the CORRECTED cycles; the     */
+/* per-row arrays hold the first pass), plus cycles1[j-j0] = first-pass */
+/* cycles, corr_len[j-j0] = rows of sub-trace j re-simulated by j-1,    */
+/* corr_lat[3i..] / corr_k[i] = the re-simulation's (f,c,s) and context */
+/* count for each re-simulated row i (untouched elsewhere).             */
+/* ------------------------------------------------------------------ */
+static long rank_of(long j, long N, long G) {
+    for (long g = 0; g < G; g++)
+        if (j < (long)(((__int128)(g + 1) * N) / G)) return g;
+    return G - 1;
+}
+
+/* one instruction: build input, predict (or take the forced latencies),
+ * update the queue.  Returns the context count k; fills f/c/s and y. */
+static int oracle_step(int arch, int mode, const double* We, double* X, oracle_queue* q,
+                       const uint8_t* trace, long row_stride, const uint16_t* forced_lat, int64_t i,
+                       int* lat3, double* y) {
+    int k = oracle_build_input(q, trace, row_stride, (long)i, X);
+    y[0] = y[1] = y[2] = 0.0;
+    if (forced_lat) {
+        lat3[0] = forced_lat[3 * i]; lat3[1] = forced_lat[3 * i + 1]; lat3[2] = forced_lat[3 * i + 2];
+    } else {
+        if (forward(arch, mode, We, X, y) != 0) return -1;
+        for (int o = 0; o < 3; o++) lat3[o] = oracle_round_latency(y[o]);
+    }
+    oracle_queue_update(q, (long)i, lat3[0], lat3[1], lat3[2], NULL, NULL, NULL);
+    return k;
+}
+
+int oracle_simulate_pec(int arch, int mode, const float* weights, long n_weights,
+                        const uint8_t* trace, long row_stride, long L, long N, long W, int cap,
+                        const uint16_t* forced_lat, long j0, long nj, long G, long limit,
+                        int64_t* cycles, int64_t* cycles1, int64_t* boundary, int32_t* corr_len,
+                        uint16_t* lat_out, int32_t* k_out, int64_t* clock_out,
+                        uint16_t* corr_lat, int32_t* corr_k, int64_t* stalls_out) {
+    if (N <= 0 || N > L || W < 0 || j0 < 0 || nj < 0 || j0 + nj > N) return -1;
+    if (cap < 1 || cap > ORACLE_MAXCAP || G < 1 || G > N || limit < 0) return -1;
+    if (!forced_lat && n_weights != oracle_arch_nparams(arch)) return -2;
+    double* X = (double*)malloc(sizeof(double) * ORACLE_ROWS * ORACLE_FEAT);
+    double* We = forced_lat ? NULL : effective_weights(arch, mode, weights, n_weights);
+    int* k1 = (int*)malloc(sizeof(int) * (size_t)(limit + 1));          /* first pass of j: k per real row */
+    int64_t* c1 = (int64_t*)malloc(sizeof(int64_t) * (size_t)(limit + 1));   /* Clock - bnd per real row */
+    oracle_queue* prev = NULL;   /* final first-pass state of sub-trace j-1 */
+    int64_t total_stalls = 0;
+    int rc = 0;
+    for (long j = j0; j < j0 + nj && rc == 0; j++) {
+        int64_t s = (int64_t)(((__int128)j * L) / N);
+        int64_t e = (int64_t)(((__int128)(j + 1) * L) / N);
+        int64_t ws = s - W > 0 ? s - W : 0;
+        /* ---- first pass of sub-trace j ---- */
+        oracle_queue* q = oracle_queue_new(cap, 0);
+        int64_t bnd = 0;
+        for (int64_t i = ws; i < e; i++) {
+            int lat3[3];
+            double y[3];
+            int k = oracle_step(arch, mode, We, X, q, trace, row_stride, forced_lat, i, lat3, y);
+            if (k < 0) { rc = -3; break; }
+            if (i == s - 1) bnd = q->clock;
+            if (i >= s) {
+                if (lat_out) for (int o = 0; o < 3; o++) lat_out[3 * i + o] = (uint16_t)lat3[o];
+                if (k_out) k_out[i] = k;
+                if (clock_out) clock_out[i] = q->clock;
+                if (i - s < limit) { k1[i - s] = k; c1[i - s] = q->clock - bnd; }
+            }
+        }
+        int64_t cyc = q->clock - bnd;
+        if (cycles1) cycles1[j - j0] = cyc;
+        if (boundary) boundary[j - j0] = bnd;
+        total_stalls += q->stalls;
+        /* ---- correction of j by j-1 ---- */
+        int32_t n_re = 0;
+        if (rc == 0 && prev && rank_of(j - 1, N, G) == rank_of(j, N, G)) {
+            oracle_queue* r = prev;                    /* j-1's final state continues */
+            const int64_t clock_start = r->clock, stalls_start = r->stalls;
+            for (int64_t i = s; i < e && i - s < limit; i++) {
+                if (r->n == k1[i - s]) break;          /* context counts match: stop */
+                int lat3[3];
+                double y[3];
+                int k = oracle_step(arch, mode, We, X, r, trace, row_stride, forced_lat, i, lat3, y);
+                if (k < 0) { rc = -3; break; }
+                if (corr_lat) for (int o = 0; o < 3; o++) corr_lat[3 * i + o] = (uint16_t)lat3[o];
+                if (corr_k) corr_k[i] = k;
+                n_re++;
+            }
+            if (n_re > 0) cyc += (r->clock - clock_start) - c1[n_re - 1];
+            total_stalls += r->stalls - stalls_start;  /* stalls of the re-simulation counted too */
+        }
+        if (corr_len) corr_len[j - j0] = n_re;
+        if (cycles) cycles[j - j0] = cyc;
+        if (prev) oracle_queue_free(prev);
+        prev = q;
+    }
+    if (prev) oracle_queue_free(prev);
+    if (stalls_out) *stalls_out = total_stalls;
+    free(X); free(We); free(k1); free(c1);
+    return rc;
+}
