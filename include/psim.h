@@ -47,6 +47,7 @@ extern "C" {
 #define PSIM_ARCH_RB7 3u  /* residual 7-conv variant (config 5, R11)                   */
 
 #define PSIM_MAX_CAP 110u /* Context_length: input length 111 = Context_length + 1 */
+#define PSIM_MAX_CORRECTION 4096u /* largest psim_opts.correction_limit (the paper uses 100, :291) */
 #define PSIM_NATTR 47u    /* trace attributes per instruction; + 3 time features = 50 (R1) */
 
 /* flags for psim_opts.flags */
@@ -83,6 +84,13 @@ typedef struct {
     uint64_t chunk_steps;   /* trace loader chunk length in lockstep steps (0 = automatic)     */
     void* stream;           /* cudaStream_t to launch on (NULL: the library creates one)       */
     uint32_t flags;         /* PSIM_RECORD_ROWS | 0                                            */
+    uint32_t correction_limit; /* post-error correction (PAPER.md:203-219 [V-B], Fig. 9; DESIGN.md
+                               R19): after the lockstep pass, every local sub-trace j except this
+                               rank's last continues from its final state over at most this many
+                               rows of sub-trace j+1, stopping at the first row whose context count
+                               matches j+1's first pass; the re-simulated cycles replace j+1's.
+                               The first sub-trace of a rank is never corrected (:219).
+                               0 = off; the paper uses 100 (:291).                              */
 } psim_opts;
 
 typedef struct {
@@ -110,6 +118,8 @@ typedef struct {
     uint64_t kernel_launches[8]; /* launches per kernel class                               */
     uint64_t layer_m[4];      /* GEMM rows per launch of layers 0..3 (M = sub-traces x positions) */
     uint32_t layer_n[4], layer_k[4];  /* GEMM N and K of layers 0..3 (device shapes)        */
+    uint64_t corrected;       /* rows re-simulated by post-error correction (0 if off)       */
+    uint64_t corr_steps;      /* lockstep steps of the correction pass                      */
 } psim_stats;
 
 /* Create a context on opts->device.  world_size > 1 with nccl_id != NULL
@@ -179,6 +189,17 @@ int psim_get_rows(const psim_ctx* ctx, uint64_t first, uint64_t n, uint16_t* out
 /* Cycles of local sub-traces [first, first + n) (index relative to this
  * rank's first sub-trace) into out (int64). */
 int psim_get_subtrace_cycles(const psim_ctx* ctx, uint64_t first, uint64_t n, int64_t* out);
+
+/* Post-error correction of local sub-traces [first, first + n) (opts.correction_limit
+ * > 0): corr_len[i] = rows of sub-trace first+i re-simulated by its predecessor
+ * (0: not corrected), cycles1[i] = its first-pass cycles (before the
+ * replacement).  Either pointer may be NULL.  STATE if correction was off. */
+int psim_get_corrections(const psim_ctx* ctx, uint64_t first, uint64_t n, int32_t* corr_len, int64_t* cycles1);
+
+/* The re-simulation's (f, c, s) and context count k of real rows
+ * [first, first + n) (requires PSIM_RECORD_ROWS and correction): rows that were
+ * not re-simulated get k = -1 and (f, c, s) = 0.  Rows outside this rank are ARG. */
+int psim_get_corrected_rows(const psim_ctx* ctx, uint64_t first, uint64_t n, uint16_t* out3, int32_t* k);
 
 /* This rank's sub-trace block [j0, j1) and trace rows [row_lo, row_hi). */
 int psim_rank_range(const psim_ctx* ctx, uint64_t* j0, uint64_t* j1, uint64_t* row_lo, uint64_t* row_hi);

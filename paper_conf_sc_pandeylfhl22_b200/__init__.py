@@ -39,7 +39,8 @@ class PsimError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("rank", ctypes.c_int), ("world_size", ctypes.c_int),
                 ("nccl_id", ctypes.c_void_p), ("queue_cap", ctypes.c_uint32), ("precision", ctypes.c_uint32),
-                ("chunk_steps", ctypes.c_uint64), ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32)]
+                ("chunk_steps", ctypes.c_uint64), ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32),
+                ("correction_limit", ctypes.c_uint32)]
 
 
 class _ModelDesc(ctypes.Structure):
@@ -53,7 +54,8 @@ class Stats(ctypes.Structure):
                 ("h2d_bytes", ctypes.c_uint64), ("gpu_launches", ctypes.c_uint64), ("sim_ms", ctypes.c_double),
                 ("load_ms", ctypes.c_double), ("local_cycles", ctypes.c_int64), ("trace_mode", ctypes.c_int32),
                 ("pad", ctypes.c_int32), ("kernel_ms", ctypes.c_double * 8), ("kernel_launches", ctypes.c_uint64 * 8),
-                ("layer_m", ctypes.c_uint64 * 4), ("layer_n", ctypes.c_uint32 * 4), ("layer_k", ctypes.c_uint32 * 4)]
+                ("layer_m", ctypes.c_uint64 * 4), ("layer_n", ctypes.c_uint32 * 4), ("layer_k", ctypes.c_uint32 * 4),
+                ("corrected", ctypes.c_uint64), ("corr_steps", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "pad"}
@@ -66,7 +68,8 @@ class Stats(ctypes.Structure):
 EXPORTS = ["psim_create", "psim_destroy", "psim_load_trace", "psim_partition", "psim_load_model",
            "psim_simulate", "psim_total_cycles", "psim_last_error", "psim_force_latencies", "psim_get_rows",
            "psim_get_subtrace_cycles", "psim_rank_range", "psim_get_stats", "psim_cnn_forward", "psim_version",
-           "psim_partition_range", "psim_kernel_class_name", "psim_nccl_unique_id"]
+           "psim_partition_range", "psim_kernel_class_name", "psim_nccl_unique_id", "psim_get_corrections",
+           "psim_get_corrected_rows"]
 
 _lib = None
 
@@ -93,6 +96,8 @@ def lib():
         L.psim_force_latencies.argtypes = [P, P, c.c_uint64]
         L.psim_get_rows.argtypes = [P, c.c_uint64, c.c_uint64, P, P, P]
         L.psim_get_subtrace_cycles.argtypes = [P, c.c_uint64, c.c_uint64, P]
+        L.psim_get_corrections.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
+        L.psim_get_corrected_rows.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
         L.psim_rank_range.argtypes = [P, c.POINTER(c.c_uint64), c.POINTER(c.c_uint64), c.POINTER(c.c_uint64),
                                       c.POINTER(c.c_uint64)]
         L.psim_get_stats.argtypes = [P, c.POINTER(Stats)]
@@ -163,7 +168,7 @@ class Simulator:
     def __init__(self, device: int = 0, precision: str = "bf16", queue_cap: int = MAX_CAP,
                  rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
                  stream=None, record_rows: bool = False, chunk_steps: int = 0, profile: bool = False,
-                 force_predict: bool = False, layerwise: bool = False):
+                 force_predict: bool = False, layerwise: bool = False, correction_limit: int = 0):
         self._keep = []
         idbuf = None
         if nccl_id is not None:
@@ -175,7 +180,8 @@ class Simulator:
                   chunk_steps=chunk_steps,
                   stream=ctypes.c_void_p(int(stream)) if stream is not None else None,
                   flags=(RECORD_ROWS if record_rows else 0) | (PROFILE if profile else 0)
-                  | (FORCE_PREDICT if force_predict else 0) | (LAYERWISE if layerwise else 0))
+                  | (FORCE_PREDICT if force_predict else 0) | (LAYERWISE if layerwise else 0),
+                  correction_limit=correction_limit)
         h = ctypes.c_void_p()
         rc = lib().psim_create(ctypes.byref(o), ctypes.byref(h))
         if rc != OK:
@@ -251,6 +257,22 @@ class Simulator:
         out = np.zeros(max(n, 1), np.int64)
         self._check(lib().psim_get_subtrace_cycles(self._h, first, n, _ptr(out)))
         return out[:n]
+
+    def corrections(self, first: int = 0, n: int | None = None):
+        """(corr_len, cycles1) of local sub-traces [first, first+n): rows re-simulated by the
+        predecessor and the first-pass cycles (post-error correction)."""
+        rr = self.rank_range()
+        n = (rr.j1 - rr.j0 - first) if n is None else n
+        cl = np.zeros(max(n, 1), np.int32)
+        c1 = np.zeros(max(n, 1), np.int64)
+        self._check(lib().psim_get_corrections(self._h, first, n, _ptr(cl), _ptr(c1)))
+        return cl[:n], c1[:n]
+
+    def get_corrected_rows(self, first: int, n: int):
+        lat = np.zeros((n, 3), np.uint16)
+        k = np.zeros(n, np.int32)
+        self._check(lib().psim_get_corrected_rows(self._h, first, n, _ptr(lat), _ptr(k)))
+        return lat, k
 
     def stats(self) -> dict:
         s = Stats()

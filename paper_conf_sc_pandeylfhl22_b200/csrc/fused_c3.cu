@@ -677,8 +677,10 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       if (lane == 0) mbar_arrive(yempty + yb);
       int pnext = 0;
       if (active) {
-        const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, first, run_head, y0, y1, y2, sHist);
-        if (a.u.step + 1 < nsteps) {
+        bool stopped = false;
+        const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, first, run_head, y0, y1, y2, sHist,
+                                                &stopped);
+        if (a.u.step + 1 < nsteps && !stopped) {
           pnext = (knew + 8) >> 3;                 // ceil((k+1)/8)
           // keep a4 rows >= P_b zero: clear the rows this sub-trace no longer computes
           for (int p = pnext; p < pb; ++p) {
@@ -807,6 +809,47 @@ __global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count,
   if (t < n) blocks[t] = (uint32_t)(t << 4);
   if (t < (n + 127) / 128) tileP[t] = 1;
   if (t == 0) { *count = (uint32_t)n; *next_count = 0; }
+}
+
+// step-0 block list of a pass that starts from existing queues (correction pass):
+// one CTA of 128 threads per 128-sub-trace tile, P_b = ceil((k+1)/8) for active b
+__global__ void __launch_bounds__(128) fused_init_state_kernel(uint64_t n, const int32_t* __restrict__ count,
+                                                                const int64_t* __restrict__ ws,
+                                                                const int64_t* __restrict__ e, uint32_t* blocks,
+                                                                uint32_t* nblocks, uint8_t* tileP) {
+  __shared__ int sSum[4], sMax[4], sBase;
+  const int m = threadIdx.x, lane = m & 31, w = m >> 5;
+  const uint64_t b = (uint64_t)blockIdx.x * 128 + m;
+  int P = 0;
+  if (b < n && e[b] > ws[b]) P = min((count[b] + 8) >> 3, 14);
+  int incl = P;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  int wmax = P;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) wmax = max(wmax, __shfl_xor_sync(0xffffffffu, wmax, o));
+  if (lane == 31) { sSum[w] = incl; sMax[w] = wmax; }
+  __syncthreads();
+  if (m == 0) {
+    const int tot = sSum[0] + sSum[1] + sSum[2] + sSum[3];
+    sBase = tot ? (int)atomicAdd(nblocks, (uint32_t)tot) : 0;
+    tileP[blockIdx.x] = (uint8_t)max(max(sMax[0], sMax[1]), max(sMax[2], sMax[3]));
+  }
+  __syncthreads();
+  int before = 0;
+  for (int q = 0; q < w; ++q) before += sSum[q];
+  const uint32_t base = (uint32_t)sBase + (uint32_t)(before + incl - P);
+  for (int p = 0; p < P; ++p) blocks[base + p] = (uint32_t)(b << 4) | (uint32_t)p;
+}
+
+void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* ws, const int64_t* e,
+                                  uint64_t n, cudaStream_t st) {
+  cudaMemsetAsync(f.count, 0, 8, st);
+  const uint64_t nt = (n + 127) / 128;
+  if (nt) fused_init_state_kernel<<<(unsigned)nt, 128, 0, st>>>(n, count, ws, e, f.blocks, f.count, f.tileP[0]);
 }
 
 // ---------------------------------------------------------------- host side

@@ -102,8 +102,36 @@ struct UpdateArgs {
   uint16_t* rec_lat;         // [rows][3] or nullptr (PSIM_RECORD_ROWS)
   int32_t* rec_k;            // [rows] or nullptr
   int64_t* rec_clock;        // [rows] or nullptr
+  // post-error correction (R19), entry-major [t][n]:
+  uint8_t* k1_rec = nullptr;   // first pass: context count at real row s_b + t, t < limit
+  uint32_t* c1_rec = nullptr;  // first pass: Clock - bnd after real row s_b + t
+  int limit = 0;
+  const uint8_t* kref = nullptr;   // correction pass: stop corrector b when its count equals
+                                   // kref[(step+1) * n + b + 1] (cycles -> st.cycles, st.e[b] = row + 1)
 };
 void launch_update(const UpdateArgs& a, cudaStream_t st);
+
+// Post-error correction state (per rank, local sub-traces; R19).  The
+// correction pass reuses the lockstep kernels on a SimState whose ws/s/e/bnd/cycles
+// point here: corrector b re-simulates rows [ws[b], e[b]) of sub-trace b+1 from
+// its own final state.
+struct Pec {
+  int limit = 0;
+  uint64_t cap = 0;             // sub-traces allocated
+  uint8_t* k1 = nullptr;        // [limit][n]
+  uint32_t* c1 = nullptr;       // [limit][n]
+  int64_t *ws = nullptr, *s = nullptr, *e = nullptr, *bnd = nullptr, *cyc = nullptr;   // [n]
+  int64_t* cycles1 = nullptr;   // [n] first-pass cycles
+  int32_t* len = nullptr;       // [n] rows of sub-trace b re-simulated by b-1
+  unsigned long long* corrected = nullptr;   // [1]
+  uint16_t* rec_lat = nullptr;  // [rows][3] re-simulated (f,c,s) (PSIM_RECORD_ROWS)
+  int32_t* rec_k = nullptr;     // [rows] re-simulated k, -1 elsewhere
+  size_t rec_cap = 0;
+};
+// set up the correction pass from the first pass's final state
+void launch_pec_init(const SimState& s, const Pec& p, cudaStream_t st);
+// cycles[b+1] = cycles1[b+1] - c1[len-1][b+1] + cyc[b] for corrected sub-traces
+void launch_pec_apply(const SimState& s, const Pec& p, cudaStream_t st);
 void launch_state_init(const SimState& s, cudaStream_t st);
 void launch_reduce_cycles(const SimState& s, cudaStream_t st);
 
@@ -151,6 +179,10 @@ struct FusedC3 {
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
 };
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
+// block list / P_tile of step 0 of a pass whose sub-traces start from a non-empty
+// queue (the correction pass): P_b = ceil((count+1)/8) for active b (ws < e)
+void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* ws, const int64_t* e,
+                                  uint64_t n, cudaStream_t st);
 // trace rows (uint8 attributes) -> bf16 operand rows of the fused conv1 layout
 void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st);
 // streamed variant for pinned host traces: the rows sub-trace b touches in lockstep

@@ -136,6 +136,8 @@ struct psim_ctx {
   int32_t* rec_k = nullptr;
   int64_t* rec_clock = nullptr;
   size_t rec_cap = 0;
+  Pec pec;                 // post-error correction (opts.correction_limit > 0)
+  bool pec_done = false;
   // results
   bool done = false;
   int64_t total = 0;
@@ -174,6 +176,7 @@ int psim_create(const psim_opts* opts, psim_ctx** out) {
   if (!opts) return PSIM_ERR_ARG;
   if (opts->world_size < 1 || opts->rank < 0 || opts->rank >= opts->world_size) return PSIM_ERR_ARG;
   if (opts->queue_cap > PSIM_MAX_CAP) return PSIM_ERR_ARG;
+  if (opts->correction_limit > PSIM_MAX_CORRECTION) return PSIM_ERR_ARG;
   if (opts->precision != PSIM_FP32 && opts->precision != PSIM_BF16) return PSIM_ERR_ARG;
   psim_ctx* ctx = new psim_ctx();
   ctx->opts = *opts;
@@ -232,6 +235,10 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->fused.tileP[0]);
   dfree(ctx->fused.tileP[1]);
   dfree(ctx->fused.a4);
+  for (void* p : {(void*)ctx->pec.k1, (void*)ctx->pec.c1, (void*)ctx->pec.ws, (void*)ctx->pec.s, (void*)ctx->pec.e,
+                  (void*)ctx->pec.bnd, (void*)ctx->pec.cyc, (void*)ctx->pec.cycles1, (void*)ctx->pec.len,
+                  (void*)ctx->pec.corrected, (void*)ctx->pec.rec_lat, (void*)ctx->pec.rec_k})
+    dfree(p);
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
@@ -587,6 +594,32 @@ static int ensure_state(psim_ctx* ctx) {
   return PSIM_OK;
 }
 
+static int ensure_pec(psim_ctx* ctx, uint64_t n, int64_t rows, bool rec) {
+  Pec& p = ctx->pec;
+  const int limit = (int)ctx->opts.correction_limit;
+  const uint64_t a = std::max<uint64_t>(n, 1);
+  if (p.cap < a || p.limit < limit) {
+    for (void* q : {(void*)p.k1, (void*)p.c1, (void*)p.ws, (void*)p.s, (void*)p.e, (void*)p.bnd, (void*)p.cyc,
+                    (void*)p.cycles1, (void*)p.len})
+      dfree(q);
+    CK(cudaMalloc(&p.k1, (size_t)limit * a + 16));
+    CK(cudaMalloc(&p.c1, (size_t)limit * a * 4 + 16));
+    CK(cudaMalloc(&p.ws, a * 8)); CK(cudaMalloc(&p.s, a * 8)); CK(cudaMalloc(&p.e, a * 8));
+    CK(cudaMalloc(&p.bnd, a * 8)); CK(cudaMalloc(&p.cyc, a * 8)); CK(cudaMalloc(&p.cycles1, a * 8));
+    CK(cudaMalloc(&p.len, a * 4));
+    p.cap = a;
+  }
+  p.limit = limit;
+  if (!p.corrected) CK(cudaMalloc(&p.corrected, 8));
+  if (rec && p.rec_cap < (size_t)rows) {
+    dfree(p.rec_lat); dfree(p.rec_k);
+    CK(cudaMalloc(&p.rec_lat, rows * 6 + 8));
+    CK(cudaMalloc(&p.rec_k, rows * 4 + 8));
+    p.rec_cap = rows;
+  }
+  return PSIM_OK;
+}
+
 extern "C" int psim_simulate(psim_ctx* ctx) {
   if (!ctx) return PSIM_ERR_ARG;
   if (!ctx->have_trace || !ctx->partitioned) FAIL(PSIM_ERR_STATE, "simulate needs load_trace and partition");
@@ -668,6 +701,8 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     dtr = ctx->d_trace;
   }
   CK(cudaEventRecord(ctx->ev[1], st));
+  const bool pec = ctx->opts.correction_limit > 0 && n > 1;
+  if (pec) { rc = ensure_pec(ctx, n, rows, rec); if (rc) return rc; }
 
   pf.begin(PSIM_KC_OTHER);
   launch_state_init(ctx->st, st);
@@ -678,6 +713,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
+  if (pec) { ua.k1_rec = ctx->pec.k1; ua.c1_rec = ctx->pec.c1; ua.limit = ctx->pec.limit; }
   if (fused && n) {
     // bf16 operand rows of the rank's trace (once per run; the trace crosses HBM once more)
     const size_t t16 = (size_t)rows * 128;
@@ -714,32 +750,79 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     launch_fused_init(ctx->fused, n, st);
     pf.end(PSIM_KC_OTHER);
   }
-  for (int64_t t = 0; t < ctx->steps && n; ++t) {
-    if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
+  // one lockstep step t of a pass: gather -> CNN -> rounding -> queue update
+  auto step = [&](GatherArgs& g, UpdateArgs& u, const int64_t* e_arr, int64_t t) -> int {
     if (fused) {
-      ga.step = t;
-      ua.step = t;
+      g.step = t;
+      u.step = t;
       pf.begin(PSIM_KC_LAYER0);
-      launch_conv_stack(ctx->fused, ga, t, n, st);
+      launch_conv_stack(ctx->fused, g, t, n, st);
       pf.end(PSIM_KC_LAYER0);
       pf.begin(PSIM_KC_LAYER0 + 3);
-      launch_fc1_head(ctx->fused, ua, ctx->st.e, t, forced, st);
+      launch_fc1_head(ctx->fused, u, e_arr, t, forced, st);
       pf.end(PSIM_KC_LAYER0 + 3);
-      continue;
+      return PSIM_OK;
     }
     if (predict) {
-      ga.step = t;
+      g.step = t;
       pf.begin(PSIM_KC_GATHER);
-      if (bf16) launch_gather_bf16(ga, (__nv_bfloat16*)ctx->buf.x, st);
-      else launch_gather_f32(ga, (float*)ctx->buf.x, st);
+      if (bf16) launch_gather_bf16(g, (__nv_bfloat16*)ctx->buf.x, st);
+      else launch_gather_f32(g, (float*)ctx->buf.x, st);
       pf.end(PSIM_KC_GATHER);
-      rc = run_cnn(ctx, n);
+      const int r = run_cnn(ctx, n);
+      if (r) return r;
+    }
+    u.step = t;
+    pf.begin(PSIM_KC_UPDATE);
+    launch_update(u, st);
+    pf.end(PSIM_KC_UPDATE);
+    return PSIM_OK;
+  };
+  for (int64_t t = 0; t < ctx->steps && n; ++t) {
+    if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
+    rc = step(ga, ua, ctx->st.e, t);
+    if (rc) return rc;
+  }
+  // ---- post-error correction pass (PAPER.md:203-219 [V-B], Fig. 9; R19) ----
+  // corrector b continues from its final state over rows of sub-trace b+1 (same
+  // kernels, lockstep over correctors, at most `limit` steps), then the
+  // re-simulated cycles replace b+1's.  Local sub-traces only: the first
+  // sub-trace of this rank is never corrected (:219).
+  if (pec) {
+    Pec& p = ctx->pec;
+    pf.begin(PSIM_KC_OTHER);
+    launch_pec_init(ctx->st, p, st);
+    pf.end(PSIM_KC_OTHER);
+    SimState s2 = ctx->st;
+    s2.ws = p.ws; s2.s = p.s; s2.e = p.e; s2.bnd = p.bnd; s2.cycles = p.cyc;
+    GatherArgs g2 = ga;
+    g2.ws = p.ws; g2.e = p.e;
+    UpdateArgs u2 = ua;
+    u2.st = s2;
+    u2.k1_rec = nullptr; u2.c1_rec = nullptr;
+    u2.kref = p.k1;
+    u2.rec_lat = rec ? p.rec_lat : nullptr;
+    u2.rec_k = rec ? p.rec_k : nullptr;
+    u2.rec_clock = nullptr;
+    if (rec) {
+      CK(cudaMemsetAsync(p.rec_lat, 0, rows * 6, st));
+      CK(cudaMemsetAsync(p.rec_k, 0xFF, rows * 4, st));
+    }
+    if (fused) {
+      // a4 rows >= P_b must be zero again: the final steps of the first pass leave rows behind
+      CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
+      pf.begin(PSIM_KC_OTHER);
+      launch_fused_init_from_state(ctx->fused, ctx->st.count, p.ws, p.e, n, st);
+      pf.end(PSIM_KC_OTHER);
+    }
+    for (int64_t t = 0; t < p.limit; ++t) {
+      rc = step(g2, u2, p.e, t);
       if (rc) return rc;
     }
-    ua.step = t;
-    pf.begin(PSIM_KC_UPDATE);
-    launch_update(ua, st);
-    pf.end(PSIM_KC_UPDATE);
+    pf.begin(PSIM_KC_OTHER);
+    launch_pec_apply(ctx->st, p, st);
+    pf.end(PSIM_KC_OTHER);
+    stats.corr_steps = (uint64_t)p.limit;
   }
   pf.begin(PSIM_KC_OTHER);
   launch_reduce_cycles(ctx->st, st);
@@ -756,6 +839,8 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   CK(cudaMemcpyAsync(hist, ctx->st.k_hist, sizeof hist, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(&stalls, ctx->st.stalls, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(&ptile_sum, ctx->st.ptile_sum, 8, cudaMemcpyDeviceToHost, st));
+  unsigned long long corrected = 0;
+  if (pec) CK(cudaMemcpyAsync(&corrected, ctx->pec.corrected, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   CK(cudaGetLastError());
   float ms_all = 0, ms_load = 0;
@@ -767,7 +852,9 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   stats.steps = (uint64_t)ctx->steps;
   uint64_t sim = 0, cnt = 0;
   for (uint64_t b = 0; b < n; ++b) { sim += ctx->h_e[b] - ctx->h_ws[b]; cnt += ctx->h_e[b] - ctx->h_s[b]; }
-  stats.simulated = sim;
+  stats.corrected = corrected;
+  stats.simulated = sim + corrected;
+  ctx->pec_done = pec;
   stats.counted = cnt;
   uint64_t launches = 0;
   for (int c = 0; c < PSIM_KC_COUNT; ++c) { stats.kernel_launches[c] = pf.launches[c]; launches += pf.launches[c]; }
@@ -851,6 +938,45 @@ extern "C" int psim_get_subtrace_cycles(const psim_ctx* cctx, uint64_t first, ui
   if (first + n > ctx->j1 - ctx->j0) FAIL(PSIM_ERR_ARG, "sub-traces outside this rank");
   CK(cudaSetDevice(ctx->opts.device));
   CK(cudaMemcpy(out, ctx->st.cycles + first, n * 8, cudaMemcpyDeviceToHost));
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_corrections(const psim_ctx* cctx, uint64_t first, uint64_t n, int32_t* corr_len,
+                                    int64_t* cycles1) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (first + n > ctx->j1 - ctx->j0) FAIL(PSIM_ERR_ARG, "sub-traces outside this rank");
+  CK(cudaSetDevice(ctx->opts.device));
+  if (ctx->opts.correction_limit == 0) FAIL(PSIM_ERR_STATE, "context created with correction_limit = 0");
+  if (!ctx->pec_done) {   // a single local sub-trace: nothing re-simulated
+    if (corr_len) memset(corr_len, 0, n * 4);
+    if (cycles1 && n) CK(cudaMemcpy(cycles1, ctx->st.cycles + first, n * 8, cudaMemcpyDeviceToHost));
+    return PSIM_OK;
+  }
+  if (corr_len && n) CK(cudaMemcpy(corr_len, ctx->pec.len + first, n * 4, cudaMemcpyDeviceToHost));
+  if (cycles1 && n) CK(cudaMemcpy(cycles1, ctx->pec.cycles1 + first, n * 8, cudaMemcpyDeviceToHost));
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_corrected_rows(const psim_ctx* cctx, uint64_t first, uint64_t n, uint16_t* out3,
+                                       int32_t* k) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (!(ctx->opts.flags & PSIM_RECORD_ROWS)) FAIL(PSIM_ERR_STATE, "context created without PSIM_RECORD_ROWS");
+  if (ctx->opts.correction_limit == 0) FAIL(PSIM_ERR_STATE, "context created with correction_limit = 0");
+  const int64_t s_first = ctx->h_s.empty() ? 0 : ctx->h_s.front();
+  if ((int64_t)first < s_first || (int64_t)(first + n) > ctx->row_hi) FAIL(PSIM_ERR_ARG, "rows outside this rank");
+  if (!ctx->pec_done) {
+    if (out3) memset(out3, 0, n * 6);
+    if (k) for (uint64_t r = 0; r < n; ++r) k[r] = -1;
+    return PSIM_OK;
+  }
+  const int64_t off = (int64_t)first - ctx->row_lo;
+  CK(cudaSetDevice(ctx->opts.device));
+  if (out3) CK(cudaMemcpy(out3, ctx->pec.rec_lat + 3 * off, n * 6, cudaMemcpyDeviceToHost));
+  if (k) CK(cudaMemcpy(k, ctx->pec.rec_k + off, n * 4, cudaMemcpyDeviceToHost));
   return PSIM_OK;
 }
 

@@ -16,6 +16,30 @@ __device__ __forceinline__ int lat_round(float y) {
   return (int)r;
 }
 
+// Post-error correction bookkeeping after the update of row i (R19).
+// First pass (k1_rec): record the context count k seen at real row s_b + t and
+// Clock - bnd after it, t < limit.  Correction pass (kref): corrector b stops
+// when its new count equals the first-pass count of sub-trace b+1 at the next
+// row; its re-simulated cycles go to st.cycles[b] and st.e[b]
+// marks the end.  Returns true if the corrector stopped.
+__device__ __forceinline__ bool pec_record_or_stop(const UpdateArgs& a, uint64_t b, int64_t i, int64_t s_b,
+                                                   int64_t nsteps, int k, int knew, int64_t clock, int64_t bnd) {
+  if (a.k1_rec && i >= s_b && i - s_b < a.limit) {
+    const uint64_t o = (uint64_t)(i - s_b) * a.st.n + b;
+    a.k1_rec[o] = (uint8_t)k;
+    a.c1_rec[o] = (uint32_t)(clock - bnd);
+  }
+  if (a.kref) {
+    const int64_t t1 = a.step + 1;
+    if (t1 < nsteps && knew == (int)a.kref[(uint64_t)t1 * a.st.n + b + 1]) {
+      a.st.cycles[b] = clock - bnd;
+      a.st.e[b] = i + 1;
+      return true;
+    }
+  }
+  return false;
+}
+
 // Warp-cooperative update of sub-trace b at lockstep step a.step (caller has
 // checked the sub-trace is active).  y: the CNN's raw outputs (nullptr when
 // teacher-forced without prediction).  Returns the new context count (all lanes).
@@ -99,6 +123,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
     int64_t bnd = a.st.bnd[b];
     if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
     if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
+    pec_record_or_stop(a, b, i, s_b, nsteps, k, base, clock, bnd);
     atomicAdd(a.st.k_hist + k, 1ull);
     if (i >= s_b) {
       const int64_t r = i - a.row_lo;
@@ -133,7 +158,7 @@ __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int 
 __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
                                                       int64_t nsteps, int k, int64_t clock, const QBatch& first,
                                                       bool has_y, float y0, float y1, float y2,
-                                                      unsigned int* hist) {
+                                                      unsigned int* hist, bool* stopped = nullptr) {
   const int64_t i = ws + a.step;
   int f, c, s;
   int pf = 0, pc = 0, ps = 0;
@@ -198,6 +223,8 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
   int64_t bnd = a.st.bnd[b];
   if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
   if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
+  const bool stop = pec_record_or_stop(a, b, i, s_b, nsteps, k, w, clock, bnd);
+  if (stopped) *stopped = stop;
   atomicAdd(hist + k, 1u);
   if (i >= s_b) {
     const int64_t r = i - a.row_lo;

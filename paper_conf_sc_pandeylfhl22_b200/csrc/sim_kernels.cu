@@ -124,6 +124,44 @@ void launch_state_init(const SimState& s, cudaStream_t st) {
   state_init_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(s);
 }
 
+// ---- post-error correction (PAPER.md:203-219 [V-B]; R19) ----
+// corrector b (every local sub-trace but the last) continues from its final
+// state over rows [s_{b+1}, s_{b+1} + len) of sub-trace b+1; it does not start
+// if its count already equals b+1's first-pass count at s_{b+1}.
+__global__ void pec_init_kernel(SimState s, Pec p) {
+  const uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (b >= s.n) return;
+  p.cycles1[b] = s.cycles[b];
+  p.len[b] = 0;
+  int64_t r0 = 0, len = 0;
+  if (b + 1 < s.n) {
+    r0 = s.s[b + 1];
+    len = min((int64_t)p.limit, s.e[b + 1] - r0);
+    if (len > 0 && s.count[b] == (int)p.k1[b + 1]) len = 0;
+  }
+  p.ws[b] = r0; p.s[b] = r0; p.e[b] = r0 + len;
+  p.bnd[b] = s.clock[b];
+  p.cyc[b] = 0;
+  if (b == 0) *p.corrected = 0;
+}
+void launch_pec_init(const SimState& s, const Pec& p, cudaStream_t st) {
+  if (s.n) pec_init_kernel<<<(unsigned)((s.n + 255) / 256), 256, 0, st>>>(s, p);
+}
+
+// "The re-simulated cycles will replace the previously simulated ones"
+__global__ void pec_apply_kernel(SimState s, Pec p) {
+  const uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (b + 1 >= s.n) return;
+  const int64_t len = p.e[b] - p.ws[b];
+  if (len <= 0) return;
+  s.cycles[b + 1] = p.cycles1[b + 1] - (int64_t)p.c1[(uint64_t)(len - 1) * s.n + b + 1] + p.cyc[b];
+  p.len[b + 1] = (int32_t)len;
+  atomicAdd(p.corrected, (unsigned long long)len);
+}
+void launch_pec_apply(const SimState& s, const Pec& p, cudaStream_t st) {
+  if (s.n > 1) pec_apply_kernel<<<(unsigned)((s.n + 255) / 256), 256, 0, st>>>(s, p);
+}
+
 // total = sum_j cycles_j (int64, exact and order independent)
 __global__ void __launch_bounds__(1024) reduce_kernel(SimState s) {
   long long acc = 0;
