@@ -199,6 +199,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg (profiling runs)")
+    ap.add_argument("--correction", type=int, default=0,
+                    help="post-error correction limit (PAPER.md:203-219; the paper uses 100); 0 = off")
     args = ap.parse_args()
     cfg = CONFIGS[args.config]
     L, N, W = cfg["L"], cfg["N"], cfg["W"]
@@ -208,7 +210,8 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     config = {"workload": cfg["desc"], "instructions": L, "subtraces": N, "warmup_W": W, "cnn": cfg["arch"],
               "queue_rows": 111, "precision": cfg["precision"],
-              "l2": "inputs larger than L2 (trace %.1f GB resident in HBM)" % (L * 48 / 1e9)}
+              "l2": "inputs larger than L2 (trace %.1f GB resident in HBM)" % (L * 48 / 1e9),
+              "post_error_correction": args.correction}
 
     if args.impl == "reference":
         # the oracle as it stands, on rank 0 only, on the host cores
@@ -273,7 +276,8 @@ def main():
         return float(t.item())
 
     sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=rank, world_size=world, nccl_id=nccl_id,
-                      stream=stream.cuda_stream, profile=True, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")))
+                      stream=stream.cuda_stream, profile=True, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")),
+                      correction_limit=args.correction)
     sim.load_model(cfg["arch"], w)
 
     def timed(trace_tensor, k_steps, warm):
@@ -317,13 +321,14 @@ def main():
             "clocks": clocks}
     if rank == 0:
         line["roofline"] = roofline(stats, args.steps, cfg)
-        line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces")}
+        line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces", "corrected",
+                                               "corr_steps")}
         line["warmup_overhead"] = round(stats["simulated"] / stats["counted"] - 1, 4)
     if rank == 0 and world == 1 and not args.no_cpu:
         # cpu_baseline: the oracle as it stands on a bounded sample of the same workload,
         # plus the sampled sub-traces' cycles vs the GPU (parity sample)
         n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W)
-        gcyc = sim.subtrace_cycles()
+        gcyc = sim.corrections()[1] if args.correction else sim.subtrace_cycles()   # first-pass cycles
         errs = [abs(int(gcyc[j]) - c) / max(c, 1) for j, c in per.items()]
         line["cpu_baseline"] = {"value": n_i / t / 1e6, "unit": "MIPS", "cores": 1, "kind": "oracle",
                                 "sample": f"{len(per)} whole sub-traces ({n_i} counted instructions, W={W} warm-up "
