@@ -347,20 +347,47 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   } else if (warp == cs::WB_WARP) {   // ============================ a4 write-back
     // the 128 staged conv3 rows (256 B each) of a tile -> a4[b][p] by TMA bulk stores,
     // off the epilogues' critical path
+    // Block ids are b-major with consecutive positions, so the rows of one sub-trace
+    // form a contiguous run in the staging area AND in a4[b][p..]: one bulk copy per
+    // run (mean ~3 rows) instead of one per row -- the TMA unit's per-copy cost was
+    // on the critical path (A3 is reused by the next tile's conv2 epilogue).
+    // Lane l owns tile rows 4l..4l+3; the next 16 rows come from lanes l+1..l+4.
+    constexpr uint32_t NONE = 0xFFFFFFFFu;
     uint32_t it = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
       uint32_t ids[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const uint32_t bi = tl * cs::TILE + u * 32 + lane;
-        ids[u] = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
+        const uint32_t bi = tl * cs::TILE + 4 * lane + u;
+        ids[u] = bi < nblocks ? a.blocks[bi] : NONE;
       }
+      uint32_t nxt[16];
+#pragma unroll
+      for (int d = 1; d <= 4; ++d)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t v = __shfl_down_sync(0xffffffffu, ids[u], d);
+          nxt[(d - 1) * 4 + u] = lane + d < 32 ? v : NONE;
+        }
+      uint32_t prev = __shfl_up_sync(0xffffffffu, ids[3], 1);
+      if (lane == 0) prev = NONE;
       wait_full(stg_full, it);
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
-        if (ids[u] != 0xFFFFFFFFu)
-          bulk_s2g(a.a4 + ((uint64_t)(ids[u] >> 4) * 14 + (ids[u] & 15)) * 128,
-                   sm + cs::A3_OFF + (u * 32 + lane) * 256, 256);
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t id = ids[u];
+        const uint32_t before = u == 0 ? prev : ids[u - 1];
+        if (id == NONE || (before != NONE && (before >> 4) == (id >> 4))) continue;   // not a run start
+        int len = 1;
+        bool run = true;
+#pragma unroll
+        for (int v = u + 1; v < u + 14; ++v) {
+          const uint32_t x = v < 4 ? ids[v] : nxt[v - 4];
+          run = run && x != NONE && (x >> 4) == (id >> 4);
+          len += run ? 1 : 0;
+        }
+        bulk_s2g(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128, sm + cs::A3_OFF + (4 * lane + u) * 256,
+                 (uint32_t)len * 256);
+      }
       bulk_commit();
       bulk_wait_read();                             // staging rows consumed -> A3 reusable
       __syncwarp();
@@ -659,6 +686,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const int yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const bool inb = b < n;
+      if (q == 0) PSIM_TS(145);
       const int tileP_cur = a.tileP[tt];
       int64_t ws = 0, s_b = 0, nsteps = 0, clock = 0;
       int kb = 0;
@@ -671,6 +699,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       if (active) load_qbatch(a.u.st, b, kb, first);
       const int pb = min((kb + 8) >> 3, 14);
       wait_full(yfull + yb, it >> 1);
+      if (q == 0) PSIM_TS(146);
       const float* yrow = sY + (yb * 128 + m) * 3;
       const float y0 = yrow[0], y1 = yrow[1], y2 = yrow[2];
       __syncwarp();
@@ -690,7 +719,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
           }
         }
       }
-      if (q == 0 && grp == 0) PSIM_TS(143);
+      if (q == 0) PSIM_TS(143);
       // tile-wide scan of pnext: one atomic per tile reserves the block-list range
       int incl = pnext;
 #pragma unroll
@@ -714,7 +743,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       }
       named_bar_sync(2 + grp, 128);
       const uint32_t base = (uint32_t)sPg[8] + (uint32_t)(before + incl - pnext);
-      if (q == 0 && grp == 0) PSIM_TS(144);
+      if (q == 0) PSIM_TS(144);
       for (int p = 0; p < pnext; ++p) a.blocks_next[base + p] = (uint32_t)(b << 4) | (uint32_t)p;
       named_bar_sync(2 + grp, 128);   // sP reused by the next tile
     }

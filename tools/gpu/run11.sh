@@ -1,0 +1,6 @@
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests -x -q -m "gpu" -k "s1_teacher or residency or s3_c3_small or fused_full or pec_s1_fused" 2>&1 | tail -2
+timeout 600 python bench.py --config c3 --steps 2 --warmup 1 --no-cpu 2>&1 | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); r=d['roofline']; print('VALUE', round(d['value'],1), 'E2E', round(d['e2e']['value'],1), 'ms', d['ms_per_step'], r['frac'], r['kernels'])"
+cp tools/gpu/libpsim_timing.so paper_conf_sc_pandeylfhl22_b200/libpsim.so
+PSIM_DEBUG_TIMING=900 PSIM_DEBUG_TIMING_OUT=gpurun_out/timing_900.txt timeout 600 python bench.py --config c3 --steps 1 --warmup 0 --no-e2e --no-cpu 2>&1 | tail -1 | cut -c1-50
