@@ -18,13 +18,16 @@
 // folded into T[P] = b_fc1 + sum_{p >= P} Wfc1[:, p] c3 (R18).
 // P_b = ceil((k_b + 1) / 8).  Exact in real arithmetic; the oracle stays dense.
 //
-// conv_stack_kernel roles (416 threads): warps 0..3 = TMEM epilogues (bias,
-// ReLU, bf16) feeding the next layer's A operand in SWIZZLE_128B smem and the
-// coalesced a4 write-back; warp 4 = TMEM allocator + single-thread tcgen05.mma
-// issuer; warps 5..12 = gather (one thread per (block, row of the current conv1
-// position), all loads of a tile issued up front).  Weights W1/W2/W3
-// stay resident in smem (112 KB).  Per 128-block tile the MMA order is
-//   c1(0) c1(1) c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1) c3(1)
+// conv_stack_kernel roles (448 threads): warps 0..3 = EG-A (conv1 epilogue:
+// TMEM -> bias, ReLU, bf16 -> A2), warps 4..7 = EG-B (conv2 epilogue -> A3,
+// conv3 epilogue -> staging rows), warp 8 = TMEM allocator, lane 0 the
+// single-thread tcgen05.mma issuer, lane 1 the W3 streamer; warps 9..12 =
+// gather (cp.async of bf16 trace rows + time features straight into the
+// SWIZZLE_128B X tile); warp 13 = a4 write-back (TMA bulk stores, one per
+// sub-trace run).  W1/W2 stay resident in smem (48 KB); W3 (64 KB) is streamed
+// one K-half (32 KB) at a time from L2, alternating with the conv3 MMAs, which
+// frees a dedicated 32 KB staging buffer.  Per 128-block tile the MMA order is
+//   c1(0) c1(1) [c3(prev,1)] c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1)
 // with K-split accumulation so A2 (16 KB) and A3 (32 KB) are single buffers.
 #include "internal.h"
 #include "sim_common.cuh"
@@ -39,11 +42,13 @@ namespace cs {
 constexpr int TILE = 128;
 constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
 constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
-constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 4 atoms [128][64]
-constexpr int X_OFF = W3_OFF + 64 * 1024;    // 2 slots x 2 atoms [128][64]
+constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of W3, streamed by TMA
+                                             // (halves alternate with the conv3 MMAs, from L2)
+constexpr int X_OFF = W3_OFF + 32 * 1024;    // 2 slots x 2 atoms [128][64]
 constexpr int A2_OFF = X_OFF + 64 * 1024;    // 1 atom  [128][64]
 constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
-constexpr int BAR_OFF = A3_OFF + 32 * 1024;  // mbarriers
+constexpr int STG_OFF = A3_OFF + 32 * 1024;  // 128 staged conv3 rows (256 B each) for the write-back warp
+constexpr int BAR_OFF = STG_OFF + 32 * 1024; // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 256;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
@@ -126,9 +131,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* c3full = bars + 16;    //     commit
   uint64_t* c3empty = bars + 17;   //     4 (EG-B)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
-  uint64_t* stg_full = bars + 19;  //     4 (EG-B): conv3 rows staged in the A3 region
+  uint64_t* stg_full = bars + 19;  //     4 (EG-B): conv3 rows staged in STG
   uint64_t* stg_empty = bars + 20; //     1 (write-back warp)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 21);
+  uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
+  uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 23);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t nblocks = *a.nblocks;
@@ -145,16 +152,16 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     mbar_init(a3full, 4); mbar_init(a3empty, 1); mbar_init(c3full, 1); mbar_init(c3empty, 4);
     mbar_init(wbar, 1);
     mbar_init(stg_full, 4); mbar_init(stg_empty, 1);
+    mbar_init(w3full, 1); mbar_init(w3empty, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    // resident weights W1/W2/W3 (112 KB) by TMA, already in the SWIZZLE_128B operand layout
-    mbar_expect_tx(wbar, 112 * 1024 + 1280);
+    // resident weights W1/W2 (48 KB) by TMA, already in the SWIZZLE_128B operand layout
+    mbar_expect_tx(wbar, 48 * 1024 + 1280);
     float* sbias = reinterpret_cast<float*>(sm + cs::BIAS_OFF);
     bulk_g2s(sbias, a.b1, 256, wbar);
     bulk_g2s(sbias + 64, a.b2, 512, wbar);
     bulk_g2s(sbias + 192, a.b3, 512, wbar);
     for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W1_OFF + kc * 8192, &tmW1, wbar, kc * 64, 0);
     for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W2_OFF + kc * 16384, &tmW2, wbar, kc * 64, 0);
-    for (int kc = 0; kc < 4; ++kc) tma_load_2d(sm + cs::W3_OFF + kc * 16384, &tmW3, wbar, kc * 64, 0);
   }
   if (warp == cs::MMA_WARP) tmem_alloc(tmem_slot, cs::TMEM_COLS);
   fence_before();
@@ -201,18 +208,19 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         mma_commit(a2empty);
         if (kh == 1) mma_commit(c2full + h);
       };
-      auto c3 = [&](uint32_t it, int kh) {
+      auto c3 = [&](uint32_t it, int kh) {   // the (2 it + kh)-th conv3 MMA group uses W3 K-half kh
         PSIM_TS(16 + 2 * kh);
         wait_full(a3full, it * 2 + kh);
         if (kh == 0) wait_empty(c3empty, it);
+        wait_full(w3full, it * 2 + kh);
         PSIM_TS(17 + 2 * kh);
         fence_after();
 #pragma unroll
         for (int k = 0; k < 8; ++k)
           mma_bf16(tmem + cs::TMEM_C3, sw128_desc(sbase + cs::A3_OFF + (k >> 2) * 16384 + (k & 3) * 32),
-                   sw128_desc(sbase + cs::W3_OFF + (2 * kh + (k >> 2)) * 16384 + (k & 3) * 32), id128,
-                   (kh | k) != 0);
+                   sw128_desc(sbase + cs::W3_OFF + (k >> 2) * 16384 + (k & 3) * 32), id128, (kh | k) != 0);
         mma_commit(a3empty);
+        mma_commit(w3empty);
         if (kh == 1) mma_commit(c3full);
       };
       uint32_t it = 0;
@@ -222,7 +230,19 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         c2(it, 0, 0); c2(it, 0, 1); c1(it, 2); c1(it, 3); c3(it, 0); c2(it, 1, 0); c2(it, 1, 1);
       }
       if (it > 0) c3(it - 1, 1);
+    } else if (lane == 1) {   // ============================ W3 streamer
+      // conv3 MMA groups alternate K-halves 0, 1, 0, 1, ...; fill n waits until the
+      // MMAs of fill n-1 have finished reading the buffer, then loads half n & 1
+      uint32_t nfill = 0;
+      for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) nfill += 2;
+      for (uint32_t f = 0; f < nfill; ++f) {
+        wait_empty(w3empty, f);
+        mbar_expect_tx(w3full, 32 * 1024);
+        for (int a2 = 0; a2 < 2; ++a2)
+          tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (f & 1) + a2) * 64, 0);
+      }
     }
+    __syncwarp();
   } else if (warp < 4) {   // ============================ EG-A: conv1 epilogues (C1 -> A2)
     const int q = warp & 3;
     const int m = q * 32 + lane;                    // tile row = TMEM lane
@@ -278,7 +298,6 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         if (q == 0) PSIM_TS(57 + 4 * h);
         fence_after();
         wait_empty(a3empty, it * 2 + h);
-        if (h == 0) wait_empty(stg_empty, it);        // previous tile's staging rows written back
         if (q == 0) PSIM_TS(58 + 4 * h);
 #pragma unroll 1
         for (int cp = 0; cp < 2; ++cp) {
@@ -310,10 +329,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       }
       // C3 (128 fp32) -> relu(+b3) -> bf16 -> plain staging rows in the A3 region -> write-back warp
       if (q == 0) PSIM_TS(64);
-      wait_full(c3full, it);                          // conv3 done: A3 is free for staging
+      wait_full(c3full, it);                          // conv3 accumulated
+      wait_empty(stg_empty, it);                      // previous tile's staging rows written back
       if (q == 0) PSIM_TS(65);
       fence_after();
-      uint8_t* row = sm + cs::A3_OFF + m * 256;
+      uint8_t* row = sm + cs::STG_OFF + m * 256;
 #pragma unroll 1
       for (int cp = 0; cp < 2; ++cp) {
         uint32_t r0[32], r1[32];
@@ -385,11 +405,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           run = run && x != NONE && (x >> 4) == (id >> 4);
           len += run ? 1 : 0;
         }
-        bulk_s2g(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128, sm + cs::A3_OFF + (4 * lane + u) * 256,
+        bulk_s2g(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128, sm + cs::STG_OFF + (4 * lane + u) * 256,
                  (uint32_t)len * 256);
       }
       bulk_commit();
-      bulk_wait_read();                             // staging rows consumed -> A3 reusable
+      bulk_wait_read();                             // staging rows consumed -> STG reusable
       __syncwarp();
       if (lane == 0) mbar_arrive(stg_empty);
     }
