@@ -262,13 +262,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C1 + s * 64, r0);
           tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C1 + s * 64 + 32, r1);
           tmem_wait_ld();
-#pragma unroll
-          for (int c = 0; c < 16; ++c) {
-            pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb1[2 * c], 0.f),
-                              fmaxf(__uint_as_float(r0[2 * c + 1]) + sb1[2 * c + 1], 0.f));
-            pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb1[32 + 2 * c], 0.f),
-                                   fmaxf(__uint_as_float(r1[2 * c + 1]) + sb1[33 + 2 * c], 0.f));
-          }
+          bias_relu_pack32(r0, sb1, pk);
+          bias_relu_pack32(r1, sb1 + 32, pk + 16);
         }
         fence_before();
         __syncwarp();
@@ -306,20 +301,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
           tmem_wait_ld();
           uint8_t* atom = sm + cs::A3_OFF + cp * 16384;   // 64 channels per atom
+          uint32_t pk[32];
+          bias_relu_pack32(r0, sb2 + cp * 64, pk);
+          bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
 #pragma unroll
-          for (int c = 0; c < 4; ++c)
-            st_sw128(atom, m, c, make_uint4(
-                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 0]) + sb2[cp * 64 + 8 * c + 0], 0.f), fmaxf(__uint_as_float(r0[8 * c + 1]) + sb2[cp * 64 + 8 * c + 1], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 2]) + sb2[cp * 64 + 8 * c + 2], 0.f), fmaxf(__uint_as_float(r0[8 * c + 3]) + sb2[cp * 64 + 8 * c + 3], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 4]) + sb2[cp * 64 + 8 * c + 4], 0.f), fmaxf(__uint_as_float(r0[8 * c + 5]) + sb2[cp * 64 + 8 * c + 5], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r0[8 * c + 6]) + sb2[cp * 64 + 8 * c + 6], 0.f), fmaxf(__uint_as_float(r0[8 * c + 7]) + sb2[cp * 64 + 8 * c + 7], 0.f))));
-#pragma unroll
-          for (int c = 0; c < 4; ++c)
-            st_sw128(atom, m, 4 + c, make_uint4(
-                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 0]) + sb2[cp * 64 + 32 + 8 * c + 0], 0.f), fmaxf(__uint_as_float(r1[8 * c + 1]) + sb2[cp * 64 + 32 + 8 * c + 1], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 2]) + sb2[cp * 64 + 32 + 8 * c + 2], 0.f), fmaxf(__uint_as_float(r1[8 * c + 3]) + sb2[cp * 64 + 32 + 8 * c + 3], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 4]) + sb2[cp * 64 + 32 + 8 * c + 4], 0.f), fmaxf(__uint_as_float(r1[8 * c + 5]) + sb2[cp * 64 + 32 + 8 * c + 5], 0.f)),
-                pack_bf16(fmaxf(__uint_as_float(r1[8 * c + 6]) + sb2[cp * 64 + 32 + 8 * c + 6], 0.f), fmaxf(__uint_as_float(r1[8 * c + 7]) + sb2[cp * 64 + 32 + 8 * c + 7], 0.f))));
+          for (int c = 0; c < 8; ++c)
+            st_sw128(atom, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
         }
         fence_before();
         fence_async_smem();
@@ -341,13 +328,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64 + 32, r1);
         tmem_wait_ld();
         uint32_t pk[32];
-#pragma unroll
-        for (int c = 0; c < 16; ++c) {
-          pk[c] = pack_bf16(fmaxf(__uint_as_float(r0[2 * c]) + sb3[cp * 64 + 2 * c], 0.f),
-                            fmaxf(__uint_as_float(r0[2 * c + 1]) + sb3[cp * 64 + 2 * c + 1], 0.f));
-          pk[16 + c] = pack_bf16(fmaxf(__uint_as_float(r1[2 * c]) + sb3[cp * 64 + 32 + 2 * c], 0.f),
-                                 fmaxf(__uint_as_float(r1[2 * c + 1]) + sb3[cp * 64 + 33 + 2 * c], 0.f));
-        }
+        bias_relu_pack32(r0, sb3 + cp * 64, pk);
+        bias_relu_pack32(r1, sb3 + cp * 64 + 32, pk + 16);
 #pragma unroll
         for (int c = 0; c < 8; ++c) {   // lane-rotated chunk order: conflict-free 256-B row pitch
           const int sel = (c + m) & 7;

@@ -138,6 +138,21 @@ __device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
   asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));   // low half = a
   return r;
 }
+// relu(a), relu(b) -> bf16x2 (RNE), low half = a; relu commutes with the rounding
+__device__ __forceinline__ uint32_t pack_bf16_relu(float a, float b) {
+  uint32_t r;
+  asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  return r;
+}
+// 32 fp32 accumulator columns + 32 fp32 biases (16-byte aligned smem) -> relu -> 16 bf16x2
+__device__ __forceinline__ void bias_relu_pack32(const uint32_t (&r)[32], const float* bias, uint32_t* out) {
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const float4 bv = *reinterpret_cast<const float4*>(bias + 4 * c);
+    out[2 * c] = pack_bf16_relu(__uint_as_float(r[4 * c]) + bv.x, __uint_as_float(r[4 * c + 1]) + bv.y);
+    out[2 * c + 1] = pack_bf16_relu(__uint_as_float(r[4 * c + 2]) + bv.z, __uint_as_float(r[4 * c + 3]) + bv.w);
+  }
+}
 // 16-byte store into a K-major SWIZZLE_128B tile: row m (128 B), logical
 // 16-byte chunk c (0..7) lands in physical chunk c ^ (m & 7).
 __device__ __forceinline__ void st_sw128(uint8_t* atom, int m, int c, uint4 v) {
