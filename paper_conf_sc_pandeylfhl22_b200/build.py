@@ -25,6 +25,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-I", INCLUDE, "-I", CSRC,
                 "--expt-relaxed-constexpr", "-Xptxas", "-v"] + (["-DPSIM_TIMING"] if os.environ.get("PSIM_TIMING") else [])
+FLAGS += os.environ.get("PSIM_EXTRA_FLAGS", "").split()   # experiments only (variant builds)
 
 
 def _sources():

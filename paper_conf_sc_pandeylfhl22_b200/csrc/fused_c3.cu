@@ -65,9 +65,7 @@ struct ConvArgs {
   const int64_t* ws;
   const int64_t* clock;
   const int32_t* count;
-  const uint32_t* q_seq;
-  const uint32_t* q_fetch;
-  const uint32_t* q_cs;
+  const uint4* q;
   int64_t step;
   uint64_t qn;               // sub-traces (entry stride of the entry-major queue)
   const __nv_bfloat16* w1;   // [64][128]
@@ -330,15 +328,22 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         uint32_t pk[32];
         bias_relu_pack32(r0, sb3 + cp * 64, pk);
         bias_relu_pack32(r1, sb3 + cp * 64 + 32, pk + 16);
+        // lane-rotated chunk order (conflict-free stores at a 256-B row pitch): rotate the
+        // 8 chunks left by m & 7 in three conditional stages, then chunk c goes to (c + m) & 7
+        const int r = m & 7;
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {   // lane-rotated chunk order: conflict-free 256-B row pitch
-          const int sel = (c + m) & 7;
-          uint4 v = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        for (int st = 1; st < 8; st <<= 1) {
+          const bool sw = (r & st) != 0;
+          uint32_t t[32];
 #pragma unroll
-          for (int t = 1; t < 8; ++t)
-            if (sel == t) v = make_uint4(pk[4 * t], pk[4 * t + 1], pk[4 * t + 2], pk[4 * t + 3]);
-          *reinterpret_cast<uint4*>(row + (cp * 8 + sel) * 16) = v;
+          for (int c = 0; c < 32; ++c) t[c] = sw ? pk[(c + 4 * st) & 31] : pk[c];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) pk[c] = t[c];
         }
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+          *reinterpret_cast<uint4*>(row + (cp * 8 + ((c + r) & 7)) * 16) =
+              make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
       }
       fence_before();
       fence_async_smem();                             // staging rows are read by TMA bulk copies
@@ -420,20 +425,25 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       mt.k = -1; mt.i = 0; mt.clo = 0;
       if (mt.valid) {
         mt.k = a.count[mt.b];
-        mt.i = (uint32_t)(a.ws[mt.b] + a.step);
+        mt.i = (uint32_t)a.ws[mt.b];                   // + step at use: no arithmetic on a pending load
         mt.clo = (uint32_t)a.clock[mt.b];
       }
     };
     auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // raw queue entry of row 2j+h
       const int R = mt.p * 8 + 2 * j + h;            // input row (PAPER.md:93 row order)
       en.kind = (mt.valid && R <= mt.k) ? (R == 0 ? 1 : 2) : 0;
-      en.seq = mt.i; en.fet = 0; en.csv = 0;         // R == 0: current instruction first
+      en.seq = mt.i + (uint32_t)a.step; en.fet = 0; en.csv = 0;   // R == 0: current instruction first (:127)
       if (en.kind == 2) {
         const uint64_t qo = (uint64_t)(mt.k - R) * a.qn + mt.b;   // context newest first (R6)
-        en.seq = a.q_seq[qo]; en.fet = a.q_fetch[qo]; en.csv = a.q_cs[qo];
+        const uint4 v = a.q[qo];
+        en.seq = v.x; en.fet = v.y; en.csv = v.z;
       }
     };
-    auto issue = [&](const Ent& en, uint32_t clo, uint8_t* atom) {   // one input row -> row m of an X atom
+    // One input row -> row m of an X atom, owner part: the time features (chunk 6) or,
+    // for a padding row, zeros in chunks 0..6.  Returns the trace16 row offset the
+    // attribute chunks 0..5 are copied from (NONE for padding).
+    constexpr uint32_t NONE = 0xFFFFFFFFu;
+    auto own = [&](const Ent& en, uint32_t clo, uint8_t* atom) -> uint32_t {
       if (en.kind) {
         int t0 = 0, t1 = 0, t2 = 0;
         if (en.kind == 2) {                          // time relative to Clock (R2)
@@ -441,14 +451,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           const int age = (int)(clo - en.fet);
           t0 = min(age, kTimeMax); t1 = min(max(0, c - age), kTimeMax); t2 = min(c + sv - age, kTimeMax);
         }
-        const uint8_t* src = reinterpret_cast<const uint8_t*>(a.trace16 + ((int64_t)en.seq - a.row_lo) * 64);
-#pragma unroll
-        for (int c = 0; c < 6; ++c) cp_async16(atom + m * 128 + ((c ^ (m & 7)) << 4), src + c * 16);
         st_sw128(atom, m, 6, make_uint4(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f), 0u, 0u));
-      } else {
-#pragma unroll
-        for (int c = 0; c < 7; ++c) st_sw128(atom, m, c, make_uint4(0, 0, 0, 0));
+        return (uint32_t)((int64_t)en.seq - a.row_lo);
       }
+#pragma unroll
+      for (int c = 0; c < 7; ++c) st_sw128(atom, m, c, make_uint4(0, 0, 0, 0));
+      return NONE;
     };
     // chunk 7 (cols 56..63) of every X row is always zero
 #pragma unroll
@@ -462,8 +470,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     meta_ids(blockIdx.x + gridDim.x, m1);
     meta_state(m0);
     meta_state(m1);
-    Ent ea, eb;                                       // raw queue parts of item n
+    Ent ea, eb, ea2, eb2;                             // raw queue parts of items n, n+1
     if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
+    if (n_items > 1) { stage_a(m0, 1, 0, ea2); stage_a(m0, 1, 1, eb2); }
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
@@ -474,13 +483,33 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
       wait_empty(xempty + s, it * 2 + (j >> 1));
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
-      issue(ea, m0.clo, sm + cs::X_OFF + s * 32768);
-      issue(eb, m0.clo, sm + cs::X_OFF + s * 32768 + 16384);
-      cp_async_commit();
-      if (nI + 1 < n_items) {                         // raw queue entries of item n+1
-        const Meta& mm = j == 3 ? m1 : m0;
-        stage_a(mm, (j + 1) & 3, 0, ea); stage_a(mm, (j + 1) & 3, 1, eb);
+      {
+        uint8_t* xa = sm + cs::X_OFF + s * 32768;
+        const uint32_t offA = own(ea, m0.clo, xa);
+        if (warp == cs::GATHER_WARP0) PSIM_TS(104 + 2 * j);
+        const uint32_t offB = own(eb, m0.clo, xa + 16384);
+        if (warp == cs::GATHER_WARP0) PSIM_TS(105 + 2 * j);
+        if (offA != NONE) {
+#pragma unroll
+          for (int c = 0; c < 6; ++c)
+            cp_async16(xa + m * 128 + ((c ^ (m & 7)) << 4),
+                       reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)offA * 64) + c * 16);
+        }
+        if (offB != NONE) {
+#pragma unroll
+          for (int c = 0; c < 6; ++c)
+            cp_async16(xa + 16384 + m * 128 + ((c ^ (m & 7)) << 4),
+                       reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)offB * 64) + c * 16);
+        }
       }
+      cp_async_commit();
+      if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
+      ea = ea2; eb = eb2;                             // item n+1's raw queue entries
+      if (nI + 2 < n_items) {                         // raw queue entries of item n+2
+        const Meta& mm = j >= 2 ? m1 : m0;
+        stage_a(mm, (j + 2) & 3, 0, ea2); stage_a(mm, (j + 2) & 3, 1, eb2);
+      }
+      if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
       if (nI > 0) {                                   // item n-1 landed -> visible to tcgen05
         cp_async_wait<1>();
         fence_async_smem();
@@ -964,7 +993,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   a.next_count = f.count + ((step + 1) & 1);
   a.trace16 = f.trace16; a.row_lo = g.row_lo;
   a.ws = g.ws; a.clock = g.clock; a.count = g.count;
-  a.q_seq = g.q_seq; a.q_fetch = g.q_fetch; a.q_cs = g.q_cs;
+  a.q = g.q;
   a.step = step;
   a.qn = g.n;
   a.w1 = f.w1; a.w2 = f.w2; a.w3 = f.w3;

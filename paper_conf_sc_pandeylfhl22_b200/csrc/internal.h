@@ -56,10 +56,10 @@ struct SimState {
   int64_t* cycles = nullptr;    // [n] Clock_end - bnd
   int32_t* count = nullptr;     // [n] live context entries
   // queue entries are ENTRY-MAJOR: entry e of sub-trace b at [e * n + b], so the
-  // threads of a warp (consecutive sub-traces) touch consecutive words
-  uint32_t* q_seq = nullptr;    // [kQStride][n] global row index of each live entry (fetch order)
-  uint32_t* q_fetch = nullptr;  // [kQStride][n] low 32 bits of the fetch Clock
-  uint32_t* q_cs = nullptr;     // [kQStride][n] c | s << 16
+  // threads of a warp (consecutive sub-traces) touch consecutive 16-byte words, and
+  // one entry is one 16-byte load (one DRAM sector) for the gather
+  uint4* q = nullptr;           // [kQStride][n] {global row index (fetch order), low 32 bits of
+                                //  the fetch Clock, c | s << 16, 0}
   unsigned long long* k_hist = nullptr;   // [112]
   unsigned long long* stalls = nullptr;   // [1]
   unsigned long long* ptile_sum = nullptr;   // [1] fused fc1: sum of P_tile over tiles and steps
@@ -83,9 +83,7 @@ struct GatherArgs {
   const int64_t* e;
   const int64_t* clock;
   const int32_t* count;
-  const uint32_t* q_seq;
-  const uint32_t* q_fetch;
-  const uint32_t* q_cs;
+  const uint4* q;
   uint64_t n;
   int64_t step;
 };

@@ -217,7 +217,7 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->model.head_b);
   SimState& s = ctx->st;
   for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
-                  (void*)s.count, (void*)s.q_seq, (void*)s.q_fetch, (void*)s.q_cs, (void*)s.k_hist,
+                  (void*)s.count, (void*)s.q, (void*)s.k_hist,
                   (void*)s.stalls, (void*)s.total, (void*)s.ptile_sum})
     dfree(p);
   dfree(ctx->buf.x);
@@ -569,14 +569,13 @@ static int ensure_state(psim_ctx* ctx) {
   SimState& s = ctx->st;
   if (ctx->st_cap < n || !s.clock) {
     for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
-                    (void*)s.count, (void*)s.q_seq, (void*)s.q_fetch, (void*)s.q_cs})
+                    (void*)s.count, (void*)s.q})
       dfree(p);
     const uint64_t a = std::max<uint64_t>(n, 1);
     CK(cudaMalloc(&s.ws, a * 8)); CK(cudaMalloc(&s.s, a * 8)); CK(cudaMalloc(&s.e, a * 8));
     CK(cudaMalloc(&s.clock, a * 8)); CK(cudaMalloc(&s.bnd, a * 8)); CK(cudaMalloc(&s.cycles, a * 8));
     CK(cudaMalloc(&s.count, a * 4));
-    CK(cudaMalloc(&s.q_seq, a * kQStride * 4)); CK(cudaMalloc(&s.q_fetch, a * kQStride * 4));
-    CK(cudaMalloc(&s.q_cs, a * kQStride * 4));
+    CK(cudaMalloc(&s.q, a * kQStride * 16));
     ctx->st_cap = a;
   }
   if (!s.k_hist) {
@@ -709,7 +708,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   pf.end(PSIM_KC_OTHER);
   const bool bf16 = ctx->model.precision == PSIM_BF16;
   GatherArgs ga{dtr, ctx->row_lo, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e, ctx->st.clock, ctx->st.count,
-                ctx->st.q_seq, ctx->st.q_fetch, ctx->st.q_cs, n, 0};
+                ctx->st.q, n, 0};
   UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};

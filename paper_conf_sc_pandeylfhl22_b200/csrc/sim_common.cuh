@@ -63,9 +63,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
   int64_t clock = a.st.clock[b];
   const int k = a.st.count[b];
   const uint64_t qn = a.st.n;                            // entry stride (entry-major layout)
-  uint32_t* qs = a.st.q_seq + b;
-  uint32_t* qf = a.st.q_fetch + b;
-  uint32_t* qc = a.st.q_cs + b;
+  uint4* qb = a.st.q + b;
 
   clock += f;
   const uint32_t clo_push = (uint32_t)clock;
@@ -75,7 +73,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
   for (int m = 0; m < 4; ++m) {
     const int ent = lane + 32 * m;
     valid[m] = ent < k;
-    if (valid[m]) { eseq[m] = qs[ent * qn]; efet[m] = qf[ent * qn]; ecs[m] = qc[ent * qn]; }
+    if (valid[m]) { const uint4 v = qb[ent * qn]; eseq[m] = v.x; efet[m] = v.y; ecs[m] = v.z; }
     if (ent == k) {                                      // push the predicted instruction (R4)
       valid[m] = true;
       eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16);
@@ -113,7 +111,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
     const unsigned bal = __ballot_sync(0xffffffffu, keep[m]);
     if (keep[m]) {
       const uint64_t pos = (uint64_t)(base + __popc(bal & lt_mask)) * qn;
-      qs[pos] = eseq[m]; qf[pos] = efet[m]; qc[pos] = ecs[m];
+      qb[pos] = make_uint4(eseq[m], efet[m], ecs[m], 0u);
     }
     base += __popc(bal);
   }
@@ -152,7 +150,7 @@ __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int 
   const uint64_t qn = st.n;
 #pragma unroll
   for (int t = 0; t < 8; ++t)
-    if (t < k) { q.s[t] = st.q_seq[t * qn + b]; q.f[t] = st.q_fetch[t * qn + b]; q.c[t] = st.q_cs[t * qn + b]; }
+    if (t < k) { const uint4 v = st.q[t * qn + b]; q.s[t] = v.x; q.f[t] = v.y; q.c[t] = v.z; }
 }
 
 __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
@@ -171,9 +169,7 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
     f = pf; c = pc; s = ps;
   }
   const uint64_t qn = a.st.n;                              // entry-major: entry e at [e * n + b]
-  uint32_t* qs = a.st.q_seq + b;
-  uint32_t* qf = a.st.q_fetch + b;
-  uint32_t* qc = a.st.q_cs + b;
+  uint4* qb = a.st.q + b;
   clock += f;
   uint32_t clo = (uint32_t)clock;
   // push the predicted instruction (R4) as entry k, then retire.
@@ -190,7 +186,7 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
       const int e = e0 + t;
       if (e < k) {
         if (e0 == 0) { vs[t] = first.s[t]; vf[t] = first.f[t]; vc[t] = first.c[t]; }   // prefetched
-        else { vs[t] = qs[e * qn]; vf[t] = qf[e * qn]; vc[t] = qc[e * qn]; }
+        else { const uint4 v = qb[e * qn]; vs[t] = v.x; vf[t] = v.y; vc[t] = v.z; }
       } else { vs[t] = push_s; vf[t] = push_f; vc[t] = push_c; }   // e == k: the pushed entry
     }
 #pragma unroll
@@ -198,8 +194,7 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
       if (e0 + t >= n_in) break;
       const int rem = (int)(vc[t] & 0xFFFF) + (int)(vc[t] >> 16) - (int)(clo - vf[t]);   // retire - Clock
       if (rem > 0) {
-        const uint64_t o = (uint64_t)w * qn;
-        qs[o] = vs[t]; qf[o] = vf[t]; qc[o] = vc[t];
+        qb[(uint64_t)w * qn] = make_uint4(vs[t], vf[t], vc[t], 0u);
         ++w;
         dmin = min(dmin, rem);
       }
@@ -211,9 +206,9 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
     const int n2 = w;
     w = 0;
     for (int e = 0; e < n2; ++e) {
-      const uint32_t sv = qs[e * qn], fv = qf[e * qn], cv = qc[e * qn];
-      if ((int)(cv & 0xFFFF) + (int)(cv >> 16) - (int)(clo - fv) > 0) {
-        qs[w * qn] = sv; qf[w * qn] = fv; qc[w * qn] = cv; ++w;
+      const uint4 v = qb[e * qn];
+      if ((int)(v.z & 0xFFFF) + (int)(v.z >> 16) - (int)(clo - v.y) > 0) {
+        qb[w * qn] = v; ++w;
       }
     }
     atomicAdd(a.st.stalls, 1ull);

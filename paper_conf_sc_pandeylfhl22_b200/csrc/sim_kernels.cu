@@ -40,9 +40,7 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
     const int k = a.count[b];
     const uint32_t clo = (uint32_t)a.clock[b];
     T* xb = x + b * (uint64_t)(kRows * kFeatPad);
-    const uint32_t* qs = a.q_seq + b;      // entry-major: entry e at [e * n]
-    const uint32_t* qf = a.q_fetch + b;
-    const uint32_t* qc = a.q_cs + b;
+    const uint4* qb = a.q + b;             // entry-major: entry e at [e * n]
     for (int r = 0; r < kRows; ++r) {
       float v0 = 0.f, v1 = 0.f;
       if (r <= k) {
@@ -52,10 +50,11 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
           row = i;
         } else {
           const int ent = k - r;                                  // newest first
-          row = qs[ent * a.n];
-          const uint32_t cs = qc[ent * a.n];
+          const uint4 en = qb[ent * a.n];
+          row = en.x;
+          const uint32_t cs = en.z;
           const int c = cs & 0xFFFF, s = cs >> 16;
-          age = (int)(clo - qf[ent * a.n]);
+          age = (int)(clo - en.y);
           remc = max(0, c - age);
           remr = c + s - age;
           age = min(age, kTimeMax); remc = min(remc, kTimeMax); remr = min(remr, kTimeMax);
