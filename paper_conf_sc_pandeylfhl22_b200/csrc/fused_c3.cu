@@ -412,47 +412,44 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // tile t+2 are loaded at position 0 of tile t, their sub-trace state at
     // position 2, queue entries of item n+1 during item n.
     const int m = tid - cs::GATHER_WARP0 * 32;
-    struct Meta { uint32_t b; int p, k; uint32_t i, clo; bool valid; };
-    struct Ent { uint32_t seq, fet, csv; int kind; };   // kind: 0 padding, 1 current, 2 context
+    // Every load below is UNCONDITIONAL (out-of-range lanes read a clamped, valid
+    // address) and lands in a register of its own: a predicated load merged into a
+    // pre-set value would make the merge wait for the load where it is issued.
+    struct Meta { uint32_t id; int k; uint32_t i, clo; bool valid; };
+    struct Ent { uint4 v; int kind; };               // kind: 0 padding, 1 current, 2 context
     auto meta_ids = [&](uint32_t tl, Meta& mt) {         // stage 1: block id
       const uint32_t bi = tl * cs::TILE + m;
       mt.valid = tl < ntiles && bi < nblocks;
-      mt.b = mt.valid ? a.blocks[bi] : 0u;               // raw id until meta_state
+      mt.id = a.blocks[mt.valid ? bi : 0u];              // nblocks > 0 whenever this runs
     };
     auto meta_state = [&](Meta& mt) {                    // stage 2: sub-trace state
-      const uint32_t id = mt.b;
-      mt.b = id >> 4; mt.p = (int)(id & 15);
-      mt.k = -1; mt.i = 0; mt.clo = 0;
-      if (mt.valid) {
-        mt.k = a.count[mt.b];
-        mt.i = (uint32_t)a.ws[mt.b];                   // + step at use: no arithmetic on a pending load
-        mt.clo = (uint32_t)a.clock[mt.b];
-      }
+      const uint32_t b = mt.id >> 4;
+      mt.k = a.count[b];
+      mt.i = (uint32_t)a.ws[b];                          // + step at use
+      mt.clo = (uint32_t)a.clock[b];
     };
     auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // raw queue entry of row 2j+h
-      const int R = mt.p * 8 + 2 * j + h;            // input row (PAPER.md:93 row order)
+      const int R = (int)(mt.id & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
       en.kind = (mt.valid && R <= mt.k) ? (R == 0 ? 1 : 2) : 0;
-      en.seq = mt.i + (uint32_t)a.step; en.fet = 0; en.csv = 0;   // R == 0: current instruction first (:127)
-      if (en.kind == 2) {
-        const uint64_t qo = (uint64_t)(mt.k - R) * a.qn + mt.b;   // context newest first (R6)
-        const uint4 v = a.q[qo];
-        en.seq = v.x; en.fet = v.y; en.csv = v.z;
-      }
+      const int ent = en.kind == 2 ? mt.k - R : 0;        // context newest first (R6)
+      en.v = a.q[(uint64_t)ent * a.qn + (mt.id >> 4)];
     };
     // One input row -> row m of an X atom, owner part: the time features (chunk 6) or,
     // for a padding row, zeros in chunks 0..6.  Returns the trace16 row offset the
     // attribute chunks 0..5 are copied from (NONE for padding).
     constexpr uint32_t NONE = 0xFFFFFFFFu;
-    auto own = [&](const Ent& en, uint32_t clo, uint8_t* atom) -> uint32_t {
+    auto own = [&](const Ent& en, const Meta& mt, uint8_t* atom) -> uint32_t {
       if (en.kind) {
         int t0 = 0, t1 = 0, t2 = 0;
+        uint32_t seq = mt.i + (uint32_t)a.step;      // R == 0: current instruction first
         if (en.kind == 2) {                          // time relative to Clock (R2)
-          const int c = en.csv & 0xFFFF, sv = en.csv >> 16;
-          const int age = (int)(clo - en.fet);
+          const int c = en.v.z & 0xFFFF, sv = en.v.z >> 16;
+          const int age = (int)(mt.clo - en.v.y);
           t0 = min(age, kTimeMax); t1 = min(max(0, c - age), kTimeMax); t2 = min(c + sv - age, kTimeMax);
+          seq = en.v.x;
         }
         st_sw128(atom, m, 6, make_uint4(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f), 0u, 0u));
-        return (uint32_t)((int64_t)en.seq - a.row_lo);
+        return (uint32_t)((int64_t)seq - a.row_lo);
       }
 #pragma unroll
       for (int c = 0; c < 7; ++c) st_sw128(atom, m, c, make_uint4(0, 0, 0, 0));
@@ -485,9 +482,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
       {
         uint8_t* xa = sm + cs::X_OFF + s * 32768;
-        const uint32_t offA = own(ea, m0.clo, xa);
+        const uint32_t offA = own(ea, m0, xa);
         if (warp == cs::GATHER_WARP0) PSIM_TS(104 + 2 * j);
-        const uint32_t offB = own(eb, m0.clo, xa + 16384);
+        const uint32_t offB = own(eb, m0, xa + 16384);
         if (warp == cs::GATHER_WARP0) PSIM_TS(105 + 2 * j);
         if (offA != NONE) {
 #pragma unroll
