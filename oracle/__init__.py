@@ -81,6 +81,12 @@ def lib():
             P, c.c_long, c.c_long, c.c_long, c.c_long,   # forced, j0, nj, G, limit
             P, P, P, P,                         # cycles, cycles1, boundary, corr_len
             P, P, P, P, P, P]                   # lat, k, clock, corr_lat, corr_k, stalls
+        _lib.oracle_simulate_metrics.restype = c.c_int
+        _lib.oracle_simulate_metrics.argtypes = [
+            c.c_int, c.c_int, P, c.c_long,      # arch, mode, weights, n
+            P, c.c_long, c.c_long, c.c_long, c.c_long, c.c_int,  # trace, stride, L, N, W, cap
+            P, c.c_long, c.c_long, c.c_long,    # forced, j0, nj, interval
+            P, P, P, P]                         # cycles, retired, retired_st, mem_bytes
     return _lib
 
 
@@ -235,3 +241,36 @@ def simulate_pec(trace: np.ndarray, N: int, W: int, *, limit: int = 100, G: int 
     if want_rows:
         out.update(lat=lat, k=k, clock=clk, corr_lat=clat, corr_k=ck)
     return out
+
+
+def simulate_metrics(trace: np.ndarray, N: int, W: int, interval: int, *, arch: str = "C3", weights=None,
+                     mode: int = FP64, cap: int = 110, forced_lat=None, j0: int = 0, nj=None,
+                     L: int | None = None, row_offset: int = 0):
+    """Interval metrics of the partitioned simulation (PAPER.md:310-318 [VI-E]; R20).
+
+    For the counted rows of sub-traces [j0, j0+nj), per interval g of
+    ``interval`` global rows: cycles (Clock advance of the steps of its rows),
+    retired (queue entries retired in those steps), retired_st (of which
+    stores), mem_bytes (data of its loads/stores served by memory).  Returns
+    dict of int64 arrays of length ceil(L / interval) plus cpi and bw
+    (bytes/cycle) where defined.
+    """
+    trace = np.ascontiguousarray(trace, dtype=np.uint8)
+    L = trace.shape[0] + row_offset if L is None else L
+    nj = N - j0 if nj is None else nj
+    w = None if weights is None else np.ascontiguousarray(weights, dtype=np.float32)
+    forced = None if forced_lat is None else np.ascontiguousarray(forced_lat, dtype=np.uint16)
+    if interval < 1:
+        raise ValueError("interval must be >= 1")
+    ng = (L + interval - 1) // interval
+    cyc, ret, ret_st, mb = (np.zeros(ng, np.int64) for _ in range(4))
+    rc = lib().oracle_simulate_metrics(
+        ARCH.get(arch, 0), mode, _ptr(w), 0 if w is None else w.size,
+        ctypes.c_void_p(trace.ctypes.data - row_offset * trace.shape[1]), trace.shape[1], L, N, W, cap,
+        _ptr(forced), j0, nj, interval, _ptr(cyc), _ptr(ret), _ptr(ret_st), _ptr(mb))
+    if rc != 0:
+        raise ValueError(f"oracle_simulate_metrics rc={rc}")
+    with np.errstate(divide="ignore", invalid="ignore"):
+        cpi = np.where(ret > 0, cyc / np.maximum(ret, 1), np.nan)
+        bw = np.where(cyc > 0, mb / np.maximum(cyc, 1), np.nan)
+    return dict(cycles=cyc, retired=ret, retired_st=ret_st, mem_bytes=mb, cpi=cpi, bw=bw)

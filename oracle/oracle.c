@@ -526,3 +526,81 @@ int oracle_simulate_pec(int arch, int mode, const float* weights, long n_weights
     free(X); free(We); free(k1); free(c1);
     return rc;
 }
+
+/* ------------------------------------------------------------------ */
+/* Interval metrics (PAPER.md:310-318 [VI-E "Predicting Other          */
+/* Simulation Metrics"]; R20).                               */
+/*                                                                     */
+/* "the simulator tracks the instruction retire events in the          */
+/* instruction queue at a certain interval ... The CPI is then computed */
+/* as the ratio of the collective predicted instruction latency over   */
+/* the number of retired instructions for an interval" and "store      */
+/* instructions [retire out of order] ... We tracked store instructions */
+/* separately" (:316).  "the memory bandwidth is the ratio of the       */
+/* amount of data accessed from memory and the latency"; data counts    */
+/* only for load/store instructions whose trace says the data came from */
+/* memory (code 2, :314).                                               */
+/*                                                                     */
+/* Interval g holds the counted rows i (s_j <= i < e_j) with            */
+/* floor(i / interval) == g.  For each such row, processed by the step  */
+/* that predicts it:                                                   */
+/*   cycles[g]   += Clock after the step - Clock before it (f + stall)  */
+/*   retired[g]  += entries removed from the queue in that step         */
+/*   retired_st[g] += those of them that are stores (attribute 8)       */
+/*   mem_bytes[g] += 2^(attr 34) if row i is a load or store (attrs 7,8) */
+/*                   with data level (attr 14) == 2, else 0             */
+/* Warm-up rows contribute nothing (their cycles are discarded, :197).  */
+/* CPI_g = cycles[g] / retired[g]; bandwidth_g = mem_bytes[g] /        */
+/* cycles[g] (bytes per cycle).  Arrays are indexed by global interval  */
+/* g in [0, ceil(L / interval)) and ADDED to (caller zeroes them).      */
+/* Trace attribute indices: the row layout of SURVEY.md Appendix C     */
+/* (the shared file format).                                           */
+/* ------------------------------------------------------------------ */
+#define ORACLE_A_LOAD 7
+#define ORACLE_A_STORE 8
+#define ORACLE_A_DLEVEL 14
+#define ORACLE_A_LOG2SIZE 34
+
+int oracle_simulate_metrics(int arch, int mode, const float* weights, long n_weights,
+                            const uint8_t* trace, long row_stride, long L, long N, long W, int cap,
+                            const uint16_t* forced_lat, long j0, long nj, long interval,
+                            int64_t* cycles, int64_t* retired, int64_t* retired_st, int64_t* mem_bytes) {
+    if (N <= 0 || N > L || W < 0 || j0 < 0 || nj < 0 || j0 + nj > N || interval < 1) return -1;
+    if (cap < 1 || cap > ORACLE_MAXCAP) return -1;
+    if (!forced_lat && n_weights != oracle_arch_nparams(arch)) return -2;
+    double* X = (double*)malloc(sizeof(double) * ORACLE_ROWS * ORACLE_FEAT);
+    double* We = forced_lat ? NULL : effective_weights(arch, mode, weights, n_weights);
+    int64_t log_seq[2 * (ORACLE_MAXCAP + 2)], log_ret[2 * (ORACLE_MAXCAP + 2)];
+    for (long j = j0; j < j0 + nj; j++) {
+        int64_t s = (int64_t)(((__int128)j * L) / N);
+        int64_t e = (int64_t)(((__int128)(j + 1) * L) / N);
+        int64_t ws = s - W > 0 ? s - W : 0;
+        oracle_queue* q = oracle_queue_new(cap, 0);
+        for (int64_t i = ws; i < e; i++) {
+            oracle_build_input(q, trace, row_stride, (long)i, X);
+            int lat3[3];
+            double y[3] = {0, 0, 0};
+            if (forced_lat) {
+                for (int o = 0; o < 3; o++) lat3[o] = forced_lat[3 * i + o];
+            } else {
+                if (forward(arch, mode, We, X, y) != 0) { free(X); free(We); oracle_queue_free(q); return -3; }
+                for (int o = 0; o < 3; o++) lat3[o] = oracle_round_latency(y[o]);
+            }
+            const int64_t clock_before = q->clock;
+            int n_ret = oracle_queue_update(q, (long)i, lat3[0], lat3[1], lat3[2], log_seq, log_ret, NULL);
+            if (i < s) continue;                       /* warm-up row: discarded (:197) */
+            const int64_t g = i / interval;
+            cycles[g] += q->clock - clock_before;
+            retired[g] += n_ret;
+            for (int r = 0; r < n_ret; r++)
+                if (trace[(size_t)log_seq[r] * row_stride + ORACLE_A_STORE]) retired_st[g]++;
+            const uint8_t* a = trace + (size_t)i * row_stride;
+            if ((a[ORACLE_A_LOAD] || a[ORACLE_A_STORE]) && a[ORACLE_A_DLEVEL] == 2)
+                mem_bytes[g] += (int64_t)1 << a[ORACLE_A_LOG2SIZE];
+        }
+        oracle_queue_free(q);
+    }
+    free(X);
+    free(We);
+    return 0;
+}
