@@ -43,6 +43,13 @@ CONFIGS = {
                desc="config2: 1M-instruction synthetic SPEC-like trace, 1024 sub-traces, W=1000, C3 CNN, bf16"),
     "c3": dict(L=100_000_000, N=65536, W=110, arch="C3", precision="bf16", seed_off=2,
                desc="config3: 100M-instruction synthetic SPEC-like trace, 65536 sub-traces, W=110, C3 CNN, bf16"),
+    # BASELINE.json configs[4]: 1B instructions, deeper residual CNN, 8 GPUs, streamed loading.
+    # [proposal, SURVEY §8d] N = 262144, W = 1000 -> 3815 instructions per sub-trace.
+    "c5": dict(L=1_000_000_000, N=262144, W=1000, arch="RB7", precision="bf16", seed_off=4,
+               desc="config5: 1B-instruction synthetic SPEC-like trace, 262144 sub-traces, W=1000, RB7 CNN, bf16"),
+    # one GPU's share of config 5 at 8 GPUs (32768 sub-traces of 3815 instructions, W=1000)
+    "c5s": dict(L=125_000_000, N=32768, W=1000, arch="RB7", precision="bf16", seed_off=4,
+                desc="config5 per-GPU slice: 125M-instruction trace, 32768 sub-traces, W=1000, RB7 CNN, bf16"),
     # profiling stand-in: config 3's batch shape (65536 sub-traces, W=110) on a 4.2M-row
     # prefix -> 174 lockstep steps with the same per-step kernel shapes (ncu runs only)
     "c3p": dict(L=65536 * 64, N=65536, W=110, arch="C3", precision="bf16", seed_off=2,
@@ -108,7 +115,19 @@ def roofline(stats, k_steps, cfg):
     hist = np.array(stats["k_hist"], np.float64)
     kmean = float((hist * np.arange(112)).sum() / max(hist.sum(), 1))
     fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0   # fused path: conv_stack + fc1_head
-    if names[dom].startswith("gemm_layer"):
+    if cfg["arch"] == "RB7" and names[dom].startswith("gemm_layer"):
+        # layer-wise tcgen05 GEMMs, reported together (one kernel, 8 launches per step): stem
+        # 2*56*100*64 + six k3 convs 6 * 2*56*192*64 + fc1 2*3584*256 per simulated instruction
+        g = [i for i in range(len(names)) if names[i].startswith("gemm_layer")]
+        g_ms = sum(ms[i] for i in g)
+        flops = float(stats["simulated"]) * k_steps * (716800 + 6 * 1376256 + 1835008)
+        achieved = flops / (g_ms / 1e3) / 1e12
+        peak = pk["bf16_tflops_sustained"]
+        out.update(kernel="gemm_tc_kernel (all RB7 layers)", share=round(g_ms / total_ms, 4), bound="tensor",
+                   achieved=round(achieved, 2), peak=peak, unit="TFLOP/s", frac=round(achieved / peak, 4),
+                   flops_per_step=flops / k_steps, peak_source=src + " bf16 sustained")
+        avg_s = g_ms / 1e3 / max(sum(launches[i] for i in g), 1)
+    elif names[dom].startswith("gemm_layer"):
         li = int(names[dom][-1])
         M, N, K = stats["layer_m"][li], stats["layer_n"][li], stats["layer_k"][li]
         if fused and li == 0:     # conv_stack: per (sub-trace, position) block conv1 4x2x100x64 + conv2 2x2x128x128 + conv3 2x256x128

@@ -48,6 +48,8 @@ extern "C" {
 
 #define PSIM_MAX_CAP 110u /* Context_length: input length 111 = Context_length + 1 */
 #define PSIM_MAX_CORRECTION 4096u /* largest psim_opts.correction_limit (the paper uses 100, :291) */
+#define PSIM_MAX_INTERVAL 262144u /* largest psim_opts.interval (keeps a sub-trace's per-interval
+                                     Clock advance below 2^32: <= 12285 per row)                */
 #define PSIM_NATTR 47u    /* trace attributes per instruction; + 3 time features = 50 (R1) */
 
 /* flags for psim_opts.flags */
@@ -91,6 +93,14 @@ typedef struct {
                                matches j+1's first pass; the re-simulated cycles replace j+1's.
                                The first sub-trace of a rank is never corrected (:219).
                                0 = off; the paper uses 100 (:291).                              */
+    uint32_t interval;      /* interval metrics (PAPER.md:310-318 [VI-E]; R20): 0 = off,
+                               else 1..PSIM_MAX_INTERVAL trace rows per interval.  For every counted
+                               row i (warm-up rows excluded, :197) of the first pass, interval
+                               g = floor(i / interval) accumulates the Clock advance of i's step,
+                               the queue entries retired in that step, those of them that are
+                               stores (attribute 8), and 2^attr34 bytes if i is a load or store
+                               (attributes 7, 8) whose data level (attribute 14) is 2 = memory
+                               (:314).  Read with psim_get_interval_metrics.                    */
 } psim_opts;
 
 typedef struct {
@@ -202,6 +212,18 @@ int psim_get_corrections(const psim_ctx* ctx, uint64_t first, uint64_t n, int32_
 int psim_get_corrected_rows(const psim_ctx* ctx, uint64_t first, uint64_t n, uint16_t* out3, int32_t* k);
 
 /* This rank's sub-trace block [j0, j1) and trace rows [row_lo, row_hi). */
+/* Interval metrics of the last simulate (psim_opts.interval > 0; PAPER.md:310-318,
+ * DESIGN.md R20): for global intervals g = first .. first+n-1 (g < ceil(L / interval)),
+ * cycles[g] (Clock advance), retired[g] (retire events), retired_st[g] (of which
+ * stores) and mem_bytes[g] (data served by memory), summed over every sub-trace
+ * of every rank (one ncclAllReduce when the context has a communicator, else this
+ * rank's part).  CPI_g = cycles / retired, bandwidth_g = mem_bytes / cycles
+ * (bytes per cycle).  Any output pointer may be NULL.  Host arrays of n int64.
+ * Metrics come from the first pass (post-error correction does not change them).
+ * PSIM_ERR_STATE if interval was 0 or before simulate; PSIM_ERR_ARG if out of range. */
+int psim_get_interval_metrics(const psim_ctx* ctx, uint64_t first, uint64_t n, int64_t* cycles,
+                              int64_t* retired, int64_t* retired_st, int64_t* mem_bytes);
+
 int psim_rank_range(const psim_ctx* ctx, uint64_t* j0, uint64_t* j1, uint64_t* row_lo, uint64_t* row_hi);
 
 /* Pure host helper (no context, no GPU): the sub-trace block [j0, j1), trace

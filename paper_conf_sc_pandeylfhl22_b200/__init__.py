@@ -27,6 +27,7 @@ PROFILE = 2
 FORCE_PREDICT = 4
 LAYERWISE = 8
 MAX_CAP = 110
+MAX_INTERVAL = 262144   # PSIM_MAX_INTERVAL
 NATTR = 47
 
 
@@ -40,7 +41,7 @@ class _Opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("rank", ctypes.c_int), ("world_size", ctypes.c_int),
                 ("nccl_id", ctypes.c_void_p), ("queue_cap", ctypes.c_uint32), ("precision", ctypes.c_uint32),
                 ("chunk_steps", ctypes.c_uint64), ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32),
-                ("correction_limit", ctypes.c_uint32)]
+                ("correction_limit", ctypes.c_uint32), ("interval", ctypes.c_uint32)]
 
 
 class _ModelDesc(ctypes.Structure):
@@ -69,7 +70,7 @@ EXPORTS = ["psim_create", "psim_destroy", "psim_load_trace", "psim_partition", "
            "psim_simulate", "psim_total_cycles", "psim_last_error", "psim_force_latencies", "psim_get_rows",
            "psim_get_subtrace_cycles", "psim_rank_range", "psim_get_stats", "psim_cnn_forward", "psim_version",
            "psim_partition_range", "psim_kernel_class_name", "psim_nccl_unique_id", "psim_get_corrections",
-           "psim_get_corrected_rows"]
+           "psim_get_corrected_rows", "psim_get_interval_metrics"]
 
 _lib = None
 
@@ -98,6 +99,7 @@ def lib():
         L.psim_get_subtrace_cycles.argtypes = [P, c.c_uint64, c.c_uint64, P]
         L.psim_get_corrections.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
         L.psim_get_corrected_rows.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
+        L.psim_get_interval_metrics.argtypes = [P, c.c_uint64, c.c_uint64, P, P, P, P]
         L.psim_rank_range.argtypes = [P, c.POINTER(c.c_uint64), c.POINTER(c.c_uint64), c.POINTER(c.c_uint64),
                                       c.POINTER(c.c_uint64)]
         L.psim_get_stats.argtypes = [P, c.POINTER(Stats)]
@@ -168,7 +170,8 @@ class Simulator:
     def __init__(self, device: int = 0, precision: str = "bf16", queue_cap: int = MAX_CAP,
                  rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
                  stream=None, record_rows: bool = False, chunk_steps: int = 0, profile: bool = False,
-                 force_predict: bool = False, layerwise: bool = False, correction_limit: int = 0):
+                 force_predict: bool = False, layerwise: bool = False, correction_limit: int = 0,
+                 interval: int = 0):
         self._keep = []
         idbuf = None
         if nccl_id is not None:
@@ -181,13 +184,15 @@ class Simulator:
                   stream=ctypes.c_void_p(int(stream)) if stream is not None else None,
                   flags=(RECORD_ROWS if record_rows else 0) | (PROFILE if profile else 0)
                   | (FORCE_PREDICT if force_predict else 0) | (LAYERWISE if layerwise else 0),
-                  correction_limit=correction_limit)
+                  correction_limit=correction_limit, interval=interval)
         h = ctypes.c_void_p()
         rc = lib().psim_create(ctypes.byref(o), ctypes.byref(h))
         if rc != OK:
             raise PsimError(rc, "psim_create failed")
         self._h = h
         self.world_size = world_size
+        self._interval = interval
+        self._L = 0
 
     def close(self):
         if getattr(self, "_h", None):
@@ -213,6 +218,7 @@ class Simulator:
         rows, stride = int(attrs.shape[0]), int(attrs.shape[1])
         n_instr = rows + first_row if n_instr is None else n_instr
         self._trace_ref = attrs     # the library borrows the buffer until simulate returns
+        self._L = n_instr
         self._check(lib().psim_load_trace(self._h, _ptr(attrs), n_instr, first_row, rows, NATTR, stride))
 
     def partition(self, n_subtraces: int, warmup: int):
@@ -273,6 +279,21 @@ class Simulator:
         k = np.zeros(n, np.int32)
         self._check(lib().psim_get_corrected_rows(self._h, first, n, _ptr(lat), _ptr(k)))
         return lat, k
+
+    def interval_metrics(self, first: int = 0, n: int | None = None) -> dict:
+        """Interval metrics of the last simulate (interval > 0, R20):
+        int64 arrays cycles / retired / retired_st / mem_bytes for global intervals
+        [first, first+n) (default: all), plus cpi = cycles / retired and bw = mem_bytes /
+        cycles (bytes per cycle) where defined."""
+        if n is None:
+            n = max(0, -(-self._L // self._interval) - first) if getattr(self, "_interval", 0) else 0
+        out = [np.zeros(max(n, 1), np.int64) for _ in range(4)]
+        self._check(lib().psim_get_interval_metrics(self._h, first, n, *[_ptr(x) for x in out]))
+        cyc, ret, ret_st, mb = (x[:n] for x in out)
+        with np.errstate(divide="ignore", invalid="ignore"):
+            cpi = np.where(ret > 0, cyc / np.maximum(ret, 1), np.nan)
+            bw = np.where(cyc > 0, mb / np.maximum(cyc, 1), np.nan)
+        return dict(cycles=cyc, retired=ret, retired_st=ret_st, mem_bytes=mb, cpi=cpi, bw=bw)
 
     def stats(self) -> dict:
         s = Stats()

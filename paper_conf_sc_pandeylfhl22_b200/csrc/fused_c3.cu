@@ -820,7 +820,8 @@ void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfl
 __global__ void __launch_bounds__(128) load_chunk16_kernel(const uint8_t* __restrict__ host, int64_t host_first_row,
                                                            int64_t stride, const int64_t* __restrict__ ws,
                                                            const int64_t* __restrict__ e, uint64_t n, int64_t t0,
-                                                           int64_t t1, int64_t row_lo, __nv_bfloat16* __restrict__ out) {
+                                                           int64_t t1, int64_t row_lo, __nv_bfloat16* __restrict__ out,
+                                                           uint8_t* __restrict__ mrow) {
   const int lane = threadIdx.x & 31;
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
@@ -829,10 +830,21 @@ __global__ void __launch_bounds__(128) load_chunk16_kernel(const uint8_t* __rest
     const int64_t r0 = ws[b] + t0;
     const int64_t r1 = min(e[b], ws[b] + t1);
 #pragma unroll 4
-    for (int64_t rb = r0; rb < r1; rb += 10) {
+    for (int64_t rb = r0; rb < r1; rb += 10) {   // warp-uniform trip count
       const int64_t r = rb + rl;
-      if (lane < 30 && r < r1) {
-        const uint4 v = *reinterpret_cast<const uint4*>(host + (r - host_first_row) * stride + q * 16);
+      const bool own = lane < 30 && r < r1;
+      uint4 v = make_uint4(0, 0, 0, 0);
+      if (own) v = *reinterpret_cast<const uint4*>(host + (r - host_first_row) * stride + q * 16);
+      // metric code of row r (interval metrics, R20): attributes 7, 8, 14 are in
+      // segment 0 (this lane, q == 0), attribute 34 in segment 2 (lane + 2)
+      const uint32_t seg2x = __shfl_down_sync(0xffffffffu, v.x, 2);
+      if (mrow && own && q == 0) {
+        const uint32_t ld = (v.y >> 24) & 0xFFu, stv = v.z & 0xFFu, dl = (v.w >> 16) & 0xFFu;
+        const uint32_t l2 = (seg2x >> 16) & 0xFFu;
+        const uint32_t mem = ((ld | stv) != 0u && dl == 2u) ? min(l2, 62u) + 1u : 0u;
+        mrow[r - row_lo] = (uint8_t)((stv ? 0x80u : 0u) | mem);
+      }
+      if (own) {
         const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
         uint32_t o[8];
 #pragma unroll
@@ -852,12 +864,12 @@ __global__ void __launch_bounds__(128) load_chunk16_kernel(const uint8_t* __rest
 }
 void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64_t stride, const int64_t* ws,
                          const int64_t* e, uint64_t n, int64_t t0, int64_t t1, int64_t row_lo,
-                         __nv_bfloat16* trace16, cudaStream_t st) {
+                         __nv_bfloat16* trace16, uint8_t* mrow, cudaStream_t st) {
   uint64_t blocks = (n * 32 + 127) / 128;
   if (blocks > 148ull * 2) blocks = 148ull * 2;   // ~one 4-warp CTA per SM next to the compute kernels
   if (blocks < 1) blocks = 1;
   load_chunk16_kernel<<<(unsigned)blocks, 128, 0, st>>>(host_rows, host_first_row, stride, ws, e, n, t0, t1, row_lo,
-                                                         trace16);
+                                                         trace16, mrow);
 }
 
 // step-0 block list: every sub-trace has k = 0 -> P = 1

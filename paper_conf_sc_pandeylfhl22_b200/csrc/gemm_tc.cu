@@ -12,7 +12,12 @@
 //               S-stage smem ring (SWIZZLE_128B, mbarrier complete_tx)
 //   warp 1      TMEM allocator + single-thread tcgen05.mma issuer
 //               (M=128, N=BN, K=16 per instruction), commits to mbarriers
-//   warps 2..5  epilogue: tcgen05.ld 32x32b -> +bias, ReLU -> bf16/fp32 -> global
+//   warps 2..5  epilogue: tcgen05.ld 32x32b -> +bias (+ residual), ReLU -> bf16/fp32 -> global
+// Stride-1 convolutions (RB7's k = 3, pad 1 residual convs) run on the same
+// kernel with no im2col: K-block kb of tap t = kb / (Cin/64) loads the A tile
+// at row offset t - 1 (TMA zero-fills rows -1 and M), and the activations are
+// laid out with one zero pad row before and after each sub-trace's positions
+// (period P = positions + 2), which the epilogue keeps zero.
 // Two TMEM accumulators (2*BN columns) let the epilogue of tile i overlap the
 // MMAs of tile i+1.
 #include <cuda.h>
@@ -112,7 +117,8 @@ struct TcCfg {
 template <int BN>
 __global__ void __launch_bounds__(192, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const float* __restrict__ bias, void* __restrict__ C, int64_t M, int K, int relu, int c_f32) {
+                   const float* __restrict__ bias, void* __restrict__ C, int64_t M, int K, int relu, int c_f32,
+                   int taps, const __nv_bfloat16* __restrict__ resid, int pad_period) {
   using Cfg = TcCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -149,12 +155,15 @@ __global__ void __launch_bounds__(192, 1)
       uint32_t phase = 0;
       for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const int m0 = (int)(tile * kBM);
+        const int kpt = nk / taps;          // K-blocks per tap
         for (int kb = 0; kb < nk; ++kb) {
           tc::mbar_wait(empty + stage, phase ^ 1);
           uint8_t* sa = smem + stage * Cfg::STAGE;
           uint8_t* sb = sa + Cfg::A_BYTES;
           tc::mbar_expect_tx(full + stage, Cfg::STAGE);
-          tc::tma_load_2d(sa, &tmA, full + stage, kb * kBK, m0);
+          const int tap = kb / kpt;
+          // taps == 1: plain GEMM; taps == 3: rows shifted by tap - 1 (zero-filled outside [0, M))
+          tc::tma_load_2d(sa, &tmA, full + stage, (kb - tap * kpt) * kBK, m0 + (taps > 1 ? tap - 1 : 0));
           tc::tma_load_2d(sb, &tmB, full + stage, kb * kBK, 0);
           if (++stage == Cfg::STAGES) { stage = 0; phase ^= 1; }
         }
@@ -195,6 +204,11 @@ __global__ void __launch_bounds__(192, 1)
       tc::mbar_wait(tfull + acc, use & 1);
       tc::fence_after();
       const int64_t row = tile * kBM + quad * 32 + lane;
+      bool pad_row = false;
+      if (pad_period) {
+        const int pr = (int)(row % pad_period);
+        pad_row = pr == 0 || pr == pad_period - 1;
+      }
 #pragma unroll 1
       for (int c0 = 0; c0 < BN; c0 += 32) {
         uint32_t r[32];
@@ -202,9 +216,24 @@ __global__ void __launch_bounds__(192, 1)
         if (row < M) {
           float v[32];
 #pragma unroll
+          for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]) + __ldg(bias + c0 + j);
+          if (resid) {   // residual block: y = relu(x + conv_b(...)) (R11)
+            const uint4* rs = reinterpret_cast<const uint4*>(resid + row * BN + c0);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const uint4 u = __ldg(rs + j);
+              const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                v[8 * j + 2 * q] += __uint_as_float(w4[q] << 16);
+                v[8 * j + 2 * q + 1] += __uint_as_float(w4[q] & 0xFFFF0000u);
+              }
+            }
+          }
+#pragma unroll
           for (int j = 0; j < 32; ++j) {
-            v[j] = __uint_as_float(r[j]) + __ldg(bias + c0 + j);
             if (relu) v[j] = fmaxf(v[j], 0.f);
+            if (pad_row) v[j] = 0.f;
           }
           if (c_f32) {
             float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(C) + row * BN + c0);
@@ -288,7 +317,7 @@ static int num_sms() {
 
 template <int BN>
 static void launch_bn(const CUtensorMap& ma, const CUtensorMap& mb, const float* b, void* C, int64_t M, int K,
-                      bool relu, bool c_f32, cudaStream_t st) {
+                      bool relu, bool c_f32, int taps, const __nv_bfloat16* resid, int pad_period, cudaStream_t st) {
   using Cfg = TcCfg<BN>;
   static bool attr = false;
   if (!attr) {
@@ -297,20 +326,22 @@ static void launch_bn(const CUtensorMap& ma, const CUtensorMap& mb, const float*
   }
   const int64_t tiles = (M + kBM - 1) / kBM;
   const int grid = (int)std::min<int64_t>(tiles, num_sms());
-  gemm_tc_kernel<BN><<<grid, 192, Cfg::SMEM, st>>>(ma, mb, b, C, M, K, relu ? 1 : 0, c_f32 ? 1 : 0);
+  gemm_tc_kernel<BN><<<grid, 192, Cfg::SMEM, st>>>(ma, mb, b, C, M, K, relu ? 1 : 0, c_f32 ? 1 : 0, taps, resid,
+                                                   pad_period);
 }
 
 void launch_gemm_tc(const __nv_bfloat16* A, const void* Wtc, const float* b, void* C, bool c_is_f32, int64_t M,
-                    int N, int K, bool relu, cudaStream_t st) {
+                    int N, int K, bool relu, cudaStream_t st, int taps, const __nv_bfloat16* resid, int pad_period) {
   CUtensorMap ma, mb;
-  if (!make_map(&ma, A, (uint64_t)M, (uint64_t)K, kBM) || !make_map(&mb, Wtc, (uint64_t)N, (uint64_t)K, N)) {
+  if (taps < 1 || K % (taps * kBK) != 0 || (resid && (c_is_f32 || N != 64 && N != 128 && N != 256)) ||
+      !make_map(&ma, A, (uint64_t)M, (uint64_t)(K / taps), kBM) || !make_map(&mb, Wtc, (uint64_t)N, (uint64_t)K, N)) {
     // leave an error for the caller's cudaGetLastError check
     cudaLaunchKernel((const void*)nullptr, dim3(1), dim3(1), nullptr, 0, st);
     return;
   }
-  if (N == 64) launch_bn<64>(ma, mb, b, C, M, K, relu, c_is_f32, st);
-  else if (N == 128) launch_bn<128>(ma, mb, b, C, M, K, relu, c_is_f32, st);
-  else launch_bn<256>(ma, mb, b, C, M, K, relu, c_is_f32, st);
+  if (N == 64) launch_bn<64>(ma, mb, b, C, M, K, relu, c_is_f32, taps, resid, pad_period, st);
+  else if (N == 128) launch_bn<128>(ma, mb, b, C, M, K, relu, c_is_f32, taps, resid, pad_period, st);
+  else launch_bn<256>(ma, mb, b, C, M, K, relu, c_is_f32, taps, resid, pad_period, st);
 }
 
 }  // namespace psim

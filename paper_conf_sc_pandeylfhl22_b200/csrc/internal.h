@@ -30,6 +30,10 @@ struct GemmLayer {
   int K = 0, N = 0;        // reduction length, output channels
   int rows_per_item = 0;   // output positions per sub-trace (M = B * rows_per_item)
   bool relu = true;
+  int taps = 1;            // 3: stride-1 k3 conv over the pad-row layout (RB7)
+  bool block_begin = false;   // this layer's input is a residual block input x
+  bool add_block_input = false;   // y = relu(x + conv(...)) with x the block input (RB7, R11)
+  int pad_period = 0;      // output rows r with r % P in {0, P-1} are zero pad rows
   void* w = nullptr;       // device [N][K], fp32 or bf16 (K-major)
   float* bias = nullptr;   // device [N] fp32
   void* w_tc = nullptr;    // device weights pre-tiled for the tcgen05 kernel (bf16)
@@ -42,6 +46,8 @@ struct Model {
   float* head_w = nullptr;        // fc2 [3][256] fp32
   float* head_b = nullptr;        // fc2 bias [3]
   int head_in = 0;                // 256
+  int item_rows = kRows;          // device input rows per sub-trace (RB7: 116 = 2 + 112 + 2 pad rows)
+  int row_off = 0;                // first input row inside an item (RB7: 2)
   bool loaded = false;
 };
 
@@ -59,7 +65,7 @@ struct SimState {
   // threads of a warp (consecutive sub-traces) touch consecutive 16-byte words, and
   // one entry is one 16-byte load (one DRAM sector) for the gather
   uint4* q = nullptr;           // [kQStride][n] {global row index (fetch order), low 32 bits of
-                                //  the fetch Clock, c | s << 16, 0}
+                                //  the fetch Clock, c | s << 16, bit 0: store (metrics, R20)}
   unsigned long long* k_hist = nullptr;   // [112]
   unsigned long long* stalls = nullptr;   // [1]
   unsigned long long* ptile_sum = nullptr;   // [1] fused fc1: sum of P_tile over tiles and steps
@@ -69,7 +75,7 @@ struct SimState {
 struct Buffers {
   size_t bytes = 0;
   void* x = nullptr;            // gathered inputs [n][112][64] (fp32 or bf16)
-  void* act[6] = {};            // per-layer activations
+  void* act[8] = {};            // per-layer activations
   float* h = nullptr;           // fc1 output [n][256] fp32
   float* y = nullptr;           // head output [n][3] fp32
 };
@@ -86,6 +92,8 @@ struct GatherArgs {
   const uint4* q;
   uint64_t n;
   int64_t step;
+  int item_rows = kRows;     // rows per sub-trace in x (RB7: 116)
+  int row_off = 0;           // row of the current instruction inside an item (RB7: 2)
 };
 void launch_gather_f32(const GatherArgs& a, float* x, cudaStream_t st);
 void launch_gather_bf16(const GatherArgs& a, __nv_bfloat16* x, cudaStream_t st);
@@ -106,8 +114,17 @@ struct UpdateArgs {
   int limit = 0;
   const uint8_t* kref = nullptr;   // correction pass: stop corrector b when its count equals
                                    // kref[(step+1) * n + b + 1] (cycles -> st.cycles, st.e[b] = row + 1)
+  // interval metrics (R20).  mrow tags pushed entries
+  // (queue word .w bit 0 = store) whenever it is set; macc/mout nullptr = no metrics.
+  const uint8_t* mrow = nullptr;   // [rows] (row - row_lo): bit 7 store, bits 0..6 0 or 1 + log2(bytes)
+                                   // of a memory-served load/store
+  uint4* macc = nullptr;           // [n] {retired, retired stores, Clock lo at segment start, 0}
+  unsigned long long* mout = nullptr;   // [n_int][4] cycles, retired, retired stores, mem bytes
+  int64_t interval = 0;
 };
 void launch_update(const UpdateArgs& a, cudaStream_t st);
+// per-row metric codes (UpdateArgs::mrow) from device-accessible uint8 trace rows
+void launch_mrow(const uint8_t* trace, int64_t stride, int64_t rows, uint8_t* out, cudaStream_t st);
 
 // Post-error correction state (per rank, local sub-traces; R19).  The
 // correction pass reuses the lockstep kernels on a SimState whose ws/s/e/bnd/cycles
@@ -147,8 +164,12 @@ void launch_gemm_simt_bf16(const __nv_bfloat16* A, const __nv_bfloat16* W, const
 // tcgen05 GEMM (tensor cores, sm_100a): bf16 A/W, fp32 accumulate in TMEM.
 // Returns false if the shape is not supported by the tensor-core kernel.
 bool gemm_tc_supported(int N, int K);
+// taps = 3: stride-1 k3 convolution over a pad-row layout (A is [M][K/3], tap t reads
+// row m + t - 1, zero outside [0, M)); resid: bf16 [M][N] added before the ReLU;
+// pad_period > 0: output rows with row % P in {0, P-1} are written as zero.
 void launch_gemm_tc(const __nv_bfloat16* A, const void* Wtc, const float* b, void* C,
-                    bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st);
+                    bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st, int taps = 1,
+                    const __nv_bfloat16* resid = nullptr, int pad_period = 0);
 // Pre-tile a [N][K] bf16 weight for the tensor-core kernel (device -> device).
 void* pretile_weight_tc(const __nv_bfloat16* W, int N, int K, cudaStream_t st);
 
@@ -187,7 +208,7 @@ void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfl
 // steps [t0, t1) are read over PCIe (zero-copy) and written as bf16 operand rows
 void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64_t stride, const int64_t* ws,
                          const int64_t* e, uint64_t n, int64_t t0, int64_t t1, int64_t row_lo,
-                         __nv_bfloat16* trace16, cudaStream_t st);
+                         __nv_bfloat16* trace16, uint8_t* mrow, cudaStream_t st);
 void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n, cudaStream_t st);
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
                      cudaStream_t st);
@@ -196,6 +217,7 @@ bool fused_make_weight_maps(FusedC3& f);
 void fused_dump_debug();
 
 // pad/convert the caller's [B][112][50] fp32 inputs (psim_cnn_forward)
-void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st);
+void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st, int item_rows = kRows,
+                       int row_off = 0);
 
 }  // namespace psim

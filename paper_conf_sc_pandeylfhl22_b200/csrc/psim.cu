@@ -138,6 +138,14 @@ struct psim_ctx {
   size_t rec_cap = 0;
   Pec pec;                 // post-error correction (opts.correction_limit > 0)
   bool pec_done = false;
+  // interval metrics (opts.interval > 0, R20)
+  uint8_t* mrow = nullptr;             // [rows] per-row metric codes
+  size_t mrow_cap = 0;
+  uint4* macc = nullptr;               // [n] per-sub-trace segment accumulators
+  uint64_t macc_cap = 0;
+  unsigned long long* mout = nullptr;  // [n_int][4] global intervals
+  uint64_t mout_cap = 0, n_int = 0;
+  bool metrics_done = false;
   // results
   bool done = false;
   int64_t total = 0;
@@ -177,6 +185,7 @@ int psim_create(const psim_opts* opts, psim_ctx** out) {
   if (opts->world_size < 1 || opts->rank < 0 || opts->rank >= opts->world_size) return PSIM_ERR_ARG;
   if (opts->queue_cap > PSIM_MAX_CAP) return PSIM_ERR_ARG;
   if (opts->correction_limit > PSIM_MAX_CORRECTION) return PSIM_ERR_ARG;
+  if (opts->interval > PSIM_MAX_INTERVAL) return PSIM_ERR_ARG;
   if (opts->precision != PSIM_FP32 && opts->precision != PSIM_BF16) return PSIM_ERR_ARG;
   psim_ctx* ctx = new psim_ctx();
   ctx->opts = *opts;
@@ -239,6 +248,9 @@ void psim_destroy(psim_ctx* ctx) {
                   (void*)ctx->pec.bnd, (void*)ctx->pec.cyc, (void*)ctx->pec.cycles1, (void*)ctx->pec.len,
                   (void*)ctx->pec.corrected, (void*)ctx->pec.rec_lat, (void*)ctx->pec.rec_k})
     dfree(p);
+  dfree(ctx->mrow);
+  dfree(ctx->macc);
+  dfree(ctx->mout);
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   delete ctx;
@@ -344,14 +356,21 @@ int psim_partition(psim_ctx* ctx, uint64_t N, uint64_t W) {
 int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, uint64_t n_floats) {
   if (!ctx || !desc || !w) return PSIM_ERR_ARG;
   if (desc->rows != 112 || desc->features != 50) FAIL(PSIM_ERR_ARG, "model input must be 112 x 50");
-  struct L_ { int kind, cin, cout, k; };   // kind 0 conv, 1 linear
+  struct L_ { int kind, cin, cout, k; };   // kind 0 conv k=s=2, 1 linear, 2 conv k=3 s=1 pad 1
   std::vector<L_> ls;
+  const bool rb7 = desc->arch == PSIM_ARCH_RB7;
   if (desc->arch == PSIM_ARCH_M2) ls = {{0, 50, 64, 2}, {0, 64, 64, 2}, {1, 1792, 256, 0}, {1, 256, 3, 0}};
   else if (desc->arch == PSIM_ARCH_C3) ls = {{0, 50, 64, 2}, {0, 64, 128, 2}, {0, 128, 128, 2}, {1, 1792, 256, 0}, {1, 256, 3, 0}};
-  else if (desc->arch == PSIM_ARCH_RB7) FAIL(PSIM_ERR_UNSUPPORTED, "RB7 is not built in this round");
-  else FAIL(PSIM_ERR_ARG, "unknown arch %u", desc->arch);
+  else if (rb7) {
+    // stem + 3 residual blocks y = relu(x + conv_b(relu(conv_a(x)))) + fc1 3584 -> 256 + fc2 (R11)
+    ls = {{0, 50, 64, 2}};
+    for (int b = 0; b < 6; ++b) ls.push_back({2, 64, 64, 3});
+    ls.push_back({1, 3584, 256, 0});
+    ls.push_back({1, 256, 3, 0});
+    if (ctx->opts.precision != PSIM_BF16) FAIL(PSIM_ERR_UNSUPPORTED, "RB7 runs on the bf16 tensor-core path only");
+  } else FAIL(PSIM_ERR_ARG, "unknown arch %u", desc->arch);
   uint64_t need = 0;
-  for (auto& l : ls) need += (uint64_t)l.cout * l.cin * (l.kind == 0 ? l.k : 1) + l.cout;
+  for (auto& l : ls) need += (uint64_t)l.cout * l.cin * (l.kind != 1 ? l.k : 1) + l.cout;
   if (need != n_floats) FAIL(PSIM_ERR_ARG, "weight count %llu != %llu for arch %u", (unsigned long long)n_floats,
                              (unsigned long long)need, desc->arch);
   CK(cudaSetDevice(ctx->opts.device));
@@ -367,7 +386,7 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
   for (size_t li = 0; li < ls.size(); ++li) {
     const L_& l = ls[li];
     const float* W = p;
-    const float* B = p + (uint64_t)l.cout * l.cin * (l.kind == 0 ? l.k : 1);
+    const float* B = p + (uint64_t)l.cout * l.cin * (l.kind != 1 ? l.k : 1);
     p = B + l.cout;
     if (li == ls.size() - 1) {   // head: fc2 stays fp32 (R16)
       CK(cudaMalloc(&m.head_w, sizeof(float) * 3 * l.cin));
@@ -390,12 +409,37 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
           for (int t = 0; t < 2; ++t) Wk[(size_t)o * g.K + t * cin_dev + c] = W[((size_t)o * l.cin + c) * 2 + t];
       pos /= 2;
       g.rows_per_item = pos;
+      if (rb7) { g.rows_per_item = pos + 2; g.pad_period = pos + 2; }   // pad-row layout of the k3 convs
+      ch = l.cout;
+    } else if (l.kind == 2) {
+      // conv k=3, stride 1, zero pad 1 over the pad-row layout [pos + 2][C]: K index = tap * Cin + channel,
+      // tap t reads position p + t - 1 (PyTorch Conv1d definition)
+      g.K = 3 * l.cin;
+      g.N = l.cout;
+      g.taps = 3;
+      Wk.assign((size_t)g.N * g.K, 0.f);
+      for (int o = 0; o < l.cout; ++o)
+        for (int c = 0; c < l.cin; ++c)
+          for (int t = 0; t < 3; ++t) Wk[(size_t)o * g.K + t * l.cin + c] = W[((size_t)o * l.cin + c) * 3 + t];
+      g.rows_per_item = pos + 2;
+      g.pad_period = pos + 2;
+      const int conv_idx = (int)li - 1;         // 0..5: conv_a of block conv_idx/2 when even
+      g.block_begin = (conv_idx & 1) == 0;
+      g.add_block_input = (conv_idx & 1) == 1;
       ch = l.cout;
     } else {
       if (l.cin != pos * ch) FAIL(PSIM_ERR_ARG, "internal: fc1 fan-in %d != %d", l.cin, pos * ch);
-      g.K = l.cin;
       g.N = l.cout;
-      Wk.assign(W, W + (size_t)g.N * g.K);   // position-major already (R11)
+      if (rb7) {
+        // A = the pad-row layout [pos + 2][ch] flattened; pad positions get zero weights
+        g.K = (pos + 2) * ch;
+        Wk.assign((size_t)g.N * g.K, 0.f);
+        for (int o = 0; o < g.N; ++o)
+          for (int q = 0; q < pos * ch; ++q) Wk[(size_t)o * g.K + ch + q] = W[(size_t)o * l.cin + q];
+      } else {
+        g.K = l.cin;
+        Wk.assign(W, W + (size_t)g.N * g.K);   // position-major already (R11)
+      }
       g.rows_per_item = 1;
       pos = 1;
       ch = l.cout;
@@ -421,7 +465,10 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
   }
   m.arch = desc->arch;
   m.precision = ctx->opts.precision;
+  m.item_rows = rb7 ? kRows + 4 : kRows;   // RB7: 2 zero rows on each side = one zero pad position
+  m.row_off = rb7 ? 2 : 0;
   m.loaded = true;
+  ctx->buf_n = 0;                            // layer buffers depend on the architecture
   // fused padding-aware path (bf16 C3): constant table of the all-padding positions
   FusedC3& fz = ctx->fused;
   dfree(fz.T);
@@ -503,8 +550,9 @@ static int ensure_buffers(psim_ctx* ctx, uint64_t n) {
   dfree(ctx->buf.h);
   dfree(ctx->buf.y);
   ctx->buf = Buffers{};
-  CK(cudaMalloc(&ctx->buf.x, n * kRows * kFeatPad * es));
-  CK(cudaMemset(ctx->buf.x, 0, n * kRows * kFeatPad * es));
+  const size_t xr = (size_t)ctx->model.item_rows;
+  CK(cudaMalloc(&ctx->buf.x, n * xr * kFeatPad * es));
+  CK(cudaMemset(ctx->buf.x, 0, n * xr * kFeatPad * es));   // pad rows stay zero
   for (size_t li = 0; li + 1 < ctx->model.layers.size(); ++li) {
     const GemmLayer& g = ctx->model.layers[li];
     CK(cudaMalloc(&ctx->buf.act[li], n * g.rows_per_item * g.N * es));
@@ -521,19 +569,25 @@ static int run_cnn(psim_ctx* ctx, uint64_t n) {
   Prof& pf = ctx->prof;
   const bool bf16 = m.precision == PSIM_BF16;
   const void* in = ctx->buf.x;
+  const void* block_in = nullptr;
   for (size_t li = 0; li < m.layers.size(); ++li) {
     const GemmLayer& g = m.layers[li];
     const bool last = li + 1 == m.layers.size();
     void* out = last ? (void*)ctx->buf.h : ctx->buf.act[li];
     const int64_t M = (int64_t)n * g.rows_per_item;
-    pf.begin(PSIM_KC_LAYER0 + (int)li);
+    if (g.block_begin) block_in = in;
+    pf.begin(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
     if (bf16) {
-      if (g.w_tc) launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
+      if (g.taps > 1 || g.add_block_input || g.pad_period) {
+        if (!g.w_tc) FAIL(PSIM_ERR_UNSUPPORTED, "layer %zu needs the tensor-core kernel", li);
+        launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream, g.taps,
+                       g.add_block_input ? (const __nv_bfloat16*)block_in : nullptr, g.pad_period);
+      } else if (g.w_tc) launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
       else launch_gemm_simt_bf16((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream);
     } else {
       launch_gemm_simt_f32((const float*)in, (const float*)g.w, g.bias, (float*)out, M, g.N, g.K, g.relu, ctx->stream);
     }
-    pf.end(PSIM_KC_LAYER0 + (int)li);
+    pf.end(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
     in = out;
   }
   pf.begin(PSIM_KC_HEAD);
@@ -552,7 +606,8 @@ extern "C" int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float
   CK(cudaMalloc(&dX, B * kRows * kFeat * sizeof(float)));
   cudaError_t e = cudaMemcpyAsync(dX, X, B * kRows * kFeat * sizeof(float), cudaMemcpyHostToDevice, ctx->stream);
   if (e == cudaSuccess) {
-    launch_pad_inputs(dX, B, ctx->buf.x, ctx->model.precision == PSIM_BF16, ctx->stream);
+    launch_pad_inputs(dX, B, ctx->buf.x, ctx->model.precision == PSIM_BF16, ctx->stream, ctx->model.item_rows,
+                      ctx->model.row_off);
     ctx->prof.reset(false, ctx->stream);
     run_cnn(ctx, B);
     e = cudaMemcpyAsync(Y, ctx->buf.y, B * 3 * sizeof(float), cudaMemcpyDeviceToHost, ctx->stream);
@@ -674,6 +729,29 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     CK(cudaMemcpyAsync(ctx->d_forced, ctx->forced.data() + 3 * ctx->row_lo, rows * 6, cudaMemcpyHostToDevice, st));
   }
 
+  const bool metrics = ctx->opts.interval > 0;
+  ctx->metrics_done = false;
+  if (metrics) {
+    const uint64_t I = ctx->opts.interval;
+    ctx->n_int = (ctx->L + I - 1) / I;
+    if (ctx->mrow_cap < (size_t)rows) {
+      dfree(ctx->mrow); ctx->mrow = nullptr;
+      CK(cudaMalloc(&ctx->mrow, rows + 16));
+      ctx->mrow_cap = rows;
+    }
+    if (ctx->macc_cap < std::max<uint64_t>(n, 1)) {
+      dfree(ctx->macc); ctx->macc = nullptr;
+      CK(cudaMalloc(&ctx->macc, std::max<uint64_t>(n, 1) * 16));
+      ctx->macc_cap = std::max<uint64_t>(n, 1);
+    }
+    if (ctx->mout_cap < ctx->n_int) {
+      dfree(ctx->mout); ctx->mout = nullptr;
+      CK(cudaMalloc(&ctx->mout, ctx->n_int * 32));
+      ctx->mout_cap = ctx->n_int;
+    }
+    CK(cudaMemsetAsync(ctx->mout, 0, ctx->n_int * 32, st));
+  }
+
   // ---- trace: the rank's rows cross the host link once ----
   CK(cudaEventRecord(ctx->ev[0], st));
   // pinned host trace + fused path: stream it in chunks of lockstep steps, overlapped with
@@ -709,10 +787,22 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   const bool bf16 = ctx->model.precision == PSIM_BF16;
   GatherArgs ga{dtr, ctx->row_lo, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e, ctx->st.clock, ctx->st.count,
                 ctx->st.q, n, 0};
+  ga.item_rows = ctx->model.item_rows;
+  ga.row_off = ctx->model.row_off;
   UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
   if (pec) { ua.k1_rec = ctx->pec.k1; ua.c1_rec = ctx->pec.c1; ua.limit = ctx->pec.limit; }
+  if (metrics) {
+    // per-row metric codes: from the device-visible uint8 rows, or written by the
+    // streaming loader chunk by chunk (stream_load)
+    if (!stream_load && rows > 0) {
+      pf.begin(PSIM_KC_OTHER);
+      launch_mrow(dtr, (int64_t)ctx->stride, rows, ctx->mrow, st);
+      pf.end(PSIM_KC_OTHER);
+    }
+    ua.mrow = ctx->mrow; ua.macc = ctx->macc; ua.mout = ctx->mout; ua.interval = (int64_t)ctx->opts.interval;
+  }
   if (fused && n) {
     // bf16 operand rows of the rank's trace (once per run; the trace crosses HBM once more)
     const size_t t16 = (size_t)rows * 128;
@@ -734,7 +824,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       for (size_t c = 0; c < nch; ++c) {
         launch_load_chunk16(ctx->trace_devptr, (int64_t)ctx->first_row, (int64_t)ctx->stride, ctx->st.ws, ctx->st.e,
                             n, (int64_t)c * chunk, (int64_t)(c + 1) * chunk, ctx->row_lo, ctx->fused.trace16,
-                            ctx->ld_stream);
+                            metrics ? ctx->mrow : nullptr, ctx->ld_stream);
         CK(cudaEventRecord(ctx->ld_events[c], ctx->ld_stream));
       }
       pf.launches[PSIM_KC_OTHER] += nch;
@@ -800,6 +890,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     u2.st = s2;
     u2.k1_rec = nullptr; u2.c1_rec = nullptr;
     u2.kref = p.k1;
+    u2.macc = nullptr; u2.mout = nullptr;   // metrics come from the first pass (R20)
     u2.rec_lat = rec ? p.rec_lat : nullptr;
     u2.rec_k = rec ? p.rec_k : nullptr;
     u2.rec_clock = nullptr;
@@ -830,6 +921,10 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   if (ctx->comm) {
     ncclResult_t r = g_nccl.allReduce(ctx->st.total, ctx->st.total, 1, ncclInt64, ncclSum, ctx->comm, st);
     if (r != ncclSuccess) FAIL(PSIM_ERR_NCCL, "ncclAllReduce: %s", g_nccl.errStr(r));
+    if (metrics && ctx->n_int) {   // interval sums over all ranks (intervals straddle rank boundaries)
+      r = g_nccl.allReduce(ctx->mout, ctx->mout, ctx->n_int * 4, ncclUint64, ncclSum, ctx->comm, st);
+      if (r != ncclSuccess) FAIL(PSIM_ERR_NCCL, "ncclAllReduce (metrics): %s", g_nccl.errStr(r));
+    }
   }
   CK(cudaEventRecord(ctx->ev[2], st));
   long long total = 0;
@@ -889,6 +984,28 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   }
   ctx->stats = stats;
   ctx->done = true;
+  ctx->metrics_done = metrics;
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_interval_metrics(const psim_ctx* cctx, uint64_t first, uint64_t n, int64_t* cycles,
+                                         int64_t* retired, int64_t* retired_st, int64_t* mem_bytes) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (!ctx->metrics_done) FAIL(PSIM_ERR_STATE, "context created with interval = 0");
+  if (first > ctx->n_int || n > ctx->n_int - first) FAIL(PSIM_ERR_ARG, "intervals outside [0, %llu)",
+                                                          (unsigned long long)ctx->n_int);
+  if (n == 0) return PSIM_OK;
+  CK(cudaSetDevice(ctx->opts.device));
+  std::vector<unsigned long long> h(n * 4);
+  CK(cudaMemcpy(h.data(), ctx->mout + first * 4, n * 32, cudaMemcpyDeviceToHost));
+  for (uint64_t g = 0; g < n; ++g) {
+    if (cycles) cycles[g] = (int64_t)h[4 * g];
+    if (retired) retired[g] = (int64_t)h[4 * g + 1];
+    if (retired_st) retired_st[g] = (int64_t)h[4 * g + 2];
+    if (mem_bytes) mem_bytes[g] = (int64_t)h[4 * g + 3];
+  }
   return PSIM_OK;
 }
 

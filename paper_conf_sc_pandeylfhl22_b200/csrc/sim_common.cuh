@@ -40,6 +40,34 @@ __device__ __forceinline__ bool pec_record_or_stop(const UpdateArgs& a, uint64_t
   return false;
 }
 
+// Interval metrics after the update of counted row i (PAPER.md:310-318 [VI-E];
+// DESIGN.md R20): the sub-trace keeps {retired, retired stores, Clock lo at the
+// start of its current interval segment} in macc[b] and adds them to interval
+// i / I when the segment ends (last row of the interval or of the sub-trace).
+// Memory bytes are rare (memory-served loads/stores) and added at once.
+// Segment Clock advance < 2^32 for I <= PSIM_MAX_INTERVAL (<= 12285 per row).
+__device__ __forceinline__ void metrics_row(const UpdateArgs& a, uint64_t b, int64_t i, int64_t s_b,
+                                            int64_t nsteps, uint32_t clo_before, uint32_t clo_after, int nret,
+                                            int nst, uint32_t code) {
+  if (!a.macc || i < s_b) return;
+  const int64_t I = a.interval;
+  const int64_t g = i / I;
+  const int64_t r = i - g * I;
+  uint4 acc = (i == s_b || r == 0) ? make_uint4(0u, 0u, clo_before, 0u) : a.macc[b];
+  acc.x += (uint32_t)nret;
+  acc.y += (uint32_t)nst;
+  unsigned long long* o = a.mout + (uint64_t)g * 4;
+  const uint32_t lb = code & 0x7Fu;
+  if (lb) atomicAdd(o + 3, 1ull << (lb - 1));
+  if (r == I - 1 || a.step == nsteps - 1) {
+    atomicAdd(o, (unsigned long long)(uint32_t)(clo_after - acc.z));
+    if (acc.x) atomicAdd(o + 1, (unsigned long long)acc.x);
+    if (acc.y) atomicAdd(o + 2, (unsigned long long)acc.y);
+  } else {
+    a.macc[b] = acc;
+  }
+}
+
 // Warp-cooperative update of sub-trace b at lockstep step a.step (caller has
 // checked the sub-trace is active).  y: the CNN's raw outputs (nullptr when
 // teacher-forced without prediction).  Returns the new context count (all lanes).
@@ -64,19 +92,21 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
   const int k = a.st.count[b];
   const uint64_t qn = a.st.n;                            // entry stride (entry-major layout)
   uint4* qb = a.st.q + b;
+  const uint32_t code = a.mrow ? a.mrow[i - a.row_lo] : 0u;   // metrics tag of row i (R20)
+  const uint32_t clo_before = (uint32_t)clock;
 
   clock += f;
   const uint32_t clo_push = (uint32_t)clock;
-  uint32_t eseq[4], efet[4], ecs[4];
+  uint32_t eseq[4], efet[4], ecs[4], ew[4] = {0u, 0u, 0u, 0u};
   bool valid[4];
 #pragma unroll
   for (int m = 0; m < 4; ++m) {
     const int ent = lane + 32 * m;
     valid[m] = ent < k;
-    if (valid[m]) { const uint4 v = qb[ent * qn]; eseq[m] = v.x; efet[m] = v.y; ecs[m] = v.z; }
+    if (valid[m]) { const uint4 v = qb[ent * qn]; eseq[m] = v.x; efet[m] = v.y; ecs[m] = v.z; ew[m] = v.w; }
     if (ent == k) {                                      // push the predicted instruction (R4)
       valid[m] = true;
-      eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16);
+      eseq[m] = (uint32_t)i; efet[m] = clo_push; ecs[m] = (uint32_t)c | ((uint32_t)s << 16); ew[m] = code >> 7;
     }
   }
   __syncwarp();
@@ -105,15 +135,16 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
     for (int m = 0; m < 4; ++m) { keep[m] = live(m, clo); kept += __popc(__ballot_sync(0xffffffffu, keep[m])); }
     if (lane == 0) atomicAdd(a.st.stalls, 1ull);
   }
-  int base = 0;
+  int base = 0, nst = 0;
 #pragma unroll
   for (int m = 0; m < 4; ++m) {
     const unsigned bal = __ballot_sync(0xffffffffu, keep[m]);
     if (keep[m]) {
       const uint64_t pos = (uint64_t)(base + __popc(bal & lt_mask)) * qn;
-      qb[pos] = make_uint4(eseq[m], efet[m], ecs[m], 0u);
+      qb[pos] = make_uint4(eseq[m], efet[m], ecs[m], ew[m]);
     }
     base += __popc(bal);
+    if (a.macc) nst += __popc(__ballot_sync(0xffffffffu, valid[m] && !keep[m] && (ew[m] & 1u)));
   }
   if (lane == 0) {
     a.st.count[b] = base;
@@ -122,6 +153,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
     if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
     if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
     pec_record_or_stop(a, b, i, s_b, nsteps, k, base, clock, bnd);
+    metrics_row(a, b, i, s_b, nsteps, clo_before, (uint32_t)clock, k + 1 - base, nst, code);
     atomicAdd(a.st.k_hist + k, 1ull);
     if (i >= s_b) {
       const int64_t r = i - a.row_lo;
@@ -143,14 +175,14 @@ namespace psim {
 // compacts in place (write index <= read index); the rare ROB-full stall
 // (R5) re-filters the compacted entries once.  Returns the new count.
 // hist: per-CTA shared histogram of k (flushed by the caller).
-struct QBatch { uint32_t s[8], f[8], c[8]; };
+struct QBatch { uint32_t s[8], f[8], c[8], w[8]; };
 
 // first 8 entries of sub-trace b (entry-major layout), to be prefetched early
 __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int k, QBatch& q) {
   const uint64_t qn = st.n;
 #pragma unroll
   for (int t = 0; t < 8; ++t)
-    if (t < k) { const uint4 v = st.q[t * qn + b]; q.s[t] = v.x; q.f[t] = v.y; q.c[t] = v.z; }
+    if (t < k) { const uint4 v = st.q[t * qn + b]; q.s[t] = v.x; q.f[t] = v.y; q.c[t] = v.z; q.w[t] = v.w; }
 }
 
 __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
@@ -170,33 +202,38 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
   }
   const uint64_t qn = a.st.n;                              // entry-major: entry e at [e * n + b]
   uint4* qb = a.st.q + b;
+  const uint32_t code = a.mrow ? a.mrow[i - a.row_lo] : 0u;   // metrics tag of row i (R20)
+  const uint32_t clo_before = (uint32_t)clock;
   clock += f;
   uint32_t clo = (uint32_t)clock;
   // push the predicted instruction (R4) as entry k, then retire.
   // Entries are streamed in batches of 8 with all loads of a batch in flight;
   // consecutive threads (sub-traces) access consecutive words (coalesced).
-  const uint32_t push_s = (uint32_t)i, push_f = clo, push_c = (uint32_t)c | ((uint32_t)s << 16);
+  const uint32_t push_s = (uint32_t)i, push_f = clo, push_c = (uint32_t)c | ((uint32_t)s << 16),
+                 push_w = code >> 7;
   const int n_in = k + 1;
-  int w = 0;
+  int w = 0, nst = 0;
   int dmin = 0x7fffffff;   // min (retire - Clock) over kept entries
   for (int e0 = 0; e0 < n_in; e0 += 8) {
-    uint32_t vs[8], vf[8], vc[8];
+    uint32_t vs[8], vf[8], vc[8], vw[8];
 #pragma unroll
     for (int t = 0; t < 8; ++t) {
       const int e = e0 + t;
       if (e < k) {
-        if (e0 == 0) { vs[t] = first.s[t]; vf[t] = first.f[t]; vc[t] = first.c[t]; }   // prefetched
-        else { const uint4 v = qb[e * qn]; vs[t] = v.x; vf[t] = v.y; vc[t] = v.z; }
-      } else { vs[t] = push_s; vf[t] = push_f; vc[t] = push_c; }   // e == k: the pushed entry
+        if (e0 == 0) { vs[t] = first.s[t]; vf[t] = first.f[t]; vc[t] = first.c[t]; vw[t] = first.w[t]; }   // prefetched
+        else { const uint4 v = qb[e * qn]; vs[t] = v.x; vf[t] = v.y; vc[t] = v.z; vw[t] = v.w; }
+      } else { vs[t] = push_s; vf[t] = push_f; vc[t] = push_c; vw[t] = push_w; }   // e == k: the pushed entry
     }
 #pragma unroll
     for (int t = 0; t < 8; ++t) {
       if (e0 + t >= n_in) break;
       const int rem = (int)(vc[t] & 0xFFFF) + (int)(vc[t] >> 16) - (int)(clo - vf[t]);   // retire - Clock
       if (rem > 0) {
-        qb[(uint64_t)w * qn] = make_uint4(vs[t], vf[t], vc[t], 0u);
+        qb[(uint64_t)w * qn] = make_uint4(vs[t], vf[t], vc[t], vw[t]);
         ++w;
         dmin = min(dmin, rem);
+      } else {
+        nst += (int)(vw[t] & 1u);
       }
     }
   }
@@ -209,6 +246,8 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
       const uint4 v = qb[e * qn];
       if ((int)(v.z & 0xFFFF) + (int)(v.z >> 16) - (int)(clo - v.y) > 0) {
         qb[w * qn] = v; ++w;
+      } else {
+        nst += (int)(v.w & 1u);
       }
     }
     atomicAdd(a.st.stalls, 1ull);
@@ -220,6 +259,7 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
   if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;
   const bool stop = pec_record_or_stop(a, b, i, s_b, nsteps, k, w, clock, bnd);
   if (stopped) *stopped = stop;
+  metrics_row(a, b, i, s_b, nsteps, clo_before, (uint32_t)clock, k + 1 - w, nst, code);
   atomicAdd(hist + k, 1u);
   if (i >= s_b) {
     const int64_t r = i - a.row_lo;

@@ -39,7 +39,7 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
     const int64_t i = ws + a.step;
     const int k = a.count[b];
     const uint32_t clo = (uint32_t)a.clock[b];
-    T* xb = x + b * (uint64_t)(kRows * kFeatPad);
+    T* xb = x + (b * (uint64_t)a.item_rows + a.row_off) * kFeatPad;
     const uint4* qb = a.q + b;             // entry-major: entry e at [e * n]
     for (int r = 0; r < kRows; ++r) {
       float v0 = 0.f, v1 = 0.f;
@@ -110,6 +110,23 @@ __global__ void __launch_bounds__(256) update_kernel(UpdateArgs a) {
 
 void launch_update(const UpdateArgs& a, cudaStream_t st) {
   update_kernel<<<grid_for(a.st.n), 256, 0, st>>>(a);
+}
+
+// per-row metric code (R20; trace attribute layout of SURVEY.md Appendix C):
+// bit 7 = store (attr 8); bits 0..6 = 1 + log2 access size (attr 34) if the row is a
+// load or store (attrs 7, 8) whose data came from memory (attr 14 == 2)
+__device__ __forceinline__ uint8_t metric_code(uint32_t load, uint32_t store, uint32_t dlevel, uint32_t log2size) {
+  const uint32_t mem = ((load | store) != 0u && dlevel == 2u) ? min(log2size, 62u) + 1u : 0u;
+  return (uint8_t)((store ? 0x80u : 0u) | mem);
+}
+__global__ void mrow_kernel(const uint8_t* __restrict__ trace, int64_t stride, int64_t rows, uint8_t* __restrict__ out) {
+  const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (r >= rows) return;
+  const uint8_t* a = trace + r * stride;
+  out[r] = metric_code(a[7], a[8], a[14], a[34]);
+}
+void launch_mrow(const uint8_t* trace, int64_t stride, int64_t rows, uint8_t* out, cudaStream_t st) {
+  if (rows > 0) mrow_kernel<<<(unsigned)((rows + 255) / 256), 256, 0, st>>>(trace, stride, rows, out);
 }
 
 __global__ void state_init_kernel(SimState s) {
@@ -218,19 +235,22 @@ void launch_head(const float* h, const float* w, const float* b, int in, float* 
   head_kernel<<<grid_for(n), 256, 0, st>>>(h, w, b, in, y, n);
 }
 
-__global__ void pad_inputs_kernel(const float* __restrict__ X, uint64_t B, void* x, bool bf16) {
+__global__ void pad_inputs_kernel(const float* __restrict__ X, uint64_t B, void* x, bool bf16, int item_rows,
+                                  int row_off) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  const uint64_t total = B * kRows * kFeatPad;
+  const uint64_t total = B * item_rows * kFeatPad;
   if (t >= total) return;
   const int c = (int)(t % kFeatPad);
   const uint64_t br = t / kFeatPad;
-  const float v = c < kFeat ? X[br * kFeat + c] : 0.f;
+  const uint64_t b = br / item_rows;
+  const int r = (int)(br % item_rows) - row_off;   // pad rows outside [0, kRows) are zero
+  const float v = (c < kFeat && r >= 0 && r < kRows) ? X[(b * kRows + r) * kFeat + c] : 0.f;
   if (bf16) reinterpret_cast<__nv_bfloat16*>(x)[t] = __float2bfloat16_rn(v);
   else reinterpret_cast<float*>(x)[t] = v;
 }
-void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st) {
-  const uint64_t total = B * kRows * kFeatPad;
-  pad_inputs_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(X, B, x, bf16);
+void launch_pad_inputs(const float* X, uint64_t B, void* x, bool bf16, cudaStream_t st, int item_rows, int row_off) {
+  const uint64_t total = B * item_rows * kFeatPad;
+  pad_inputs_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(X, B, x, bf16, item_rows, row_off);
 }
 
 }  // namespace psim
