@@ -295,7 +295,7 @@ def main():
         return float(t.item())
 
     sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=rank, world_size=world, nccl_id=nccl_id,
-                      stream=stream.cuda_stream, profile=True, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")),
+                      stream=stream.cuda_stream, profile=os.environ.get("PSIM_NOPROF") is None, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")),
                       correction_limit=args.correction)
     sim.load_model(cfg["arch"], w)
 
@@ -339,7 +339,7 @@ def main():
             "total_cycles": total, "e2e": e2e, "gpu_launches": int(sum(stats["kernel_launches"])),
             "clocks": clocks}
     if rank == 0:
-        line["roofline"] = roofline(stats, args.steps, cfg)
+        line["roofline"] = roofline(stats, args.steps, cfg) if sum(stats["kernel_ms"]) > 0 else None
         line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces", "corrected",
                                                "corr_steps")}
         line["warmup_overhead"] = round(stats["simulated"] / stats["counted"] - 1, 4)

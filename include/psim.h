@@ -61,8 +61,11 @@ extern "C" {
                                 given trajectory, R17)                              */
 #define PSIM_LAYERWISE 8u    /* bf16 C3: use the layer-by-layer GEMM path instead of the fused
                                 padding-aware kernels (A/B comparison, parity of both)       */
-#define PSIM_PROFILE 2u      /* time every kernel class with CUDA events on the launch stream
-                                (psim_stats.kernel_ms / kernel_launches)                    */
+#define PSIM_PROFILE 2u      /* time kernel classes with CUDA events on the launch stream: every
+                                launch outside the step loop and the launches of every 16th
+                                lockstep step (events between all launches would serialise the
+                                programmatic-dependent-launch overlap of the fused kernels);
+                                psim_stats.kernel_ms is scaled to all launches of a class  */
 
 /* kernel classes reported in psim_stats.kernel_ms (names: psim_kernel_class_name) */
 #define PSIM_KC_GATHER 0

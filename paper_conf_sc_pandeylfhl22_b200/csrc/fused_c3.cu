@@ -60,7 +60,8 @@ struct ConvArgs {
   const uint32_t* blocks;    // block ids (b << 4 | p) of this step
   const uint32_t* nblocks;   // count of this step's list
   uint32_t* next_count;      // the other step parity's counter, reset here
-  const __nv_bfloat16* trace16;   // [rows][64] bf16 operand rows (attributes at cols 0..46)
+  const __nv_bfloat16* trace16;   // [rows + 1][64] bf16 operand rows (attributes at cols 0..46), row `rows` zero
+  uint32_t zero_row;         // index of the all-zero trace16 row (padding rows of the input)
   int64_t row_lo;
   const int64_t* ws;
   const int64_t* clock;
@@ -112,7 +113,7 @@ __device__ void load_weight_sw128(uint8_t* dst, const __nv_bfloat16* w, int rows
 
 __global__ void __launch_bounds__(cs::THREADS, 1)
     conv_stack_kernel(ConvArgs a, const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2,
-                      const __grid_constant__ CUtensorMap tmW3) {
+                      const __grid_constant__ CUtensorMap tmW3, const __grid_constant__ CUtensorMap tmX) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
@@ -133,16 +134,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* stg_empty = bars + 20; //     1 (write-back warp)
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 23);
+  uint64_t* xtma = bars + 23;      // [2] 4 gather warps (expect_tx) + the gathered rows (complete_tx)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 25);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const uint32_t nblocks = *a.nblocks;
-  const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
-  if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
 
   if (tid == 0) {
     for (int i = 0; i < 2; ++i) {
-      mbar_init(xfull + i, 4); mbar_init(xempty + i, 1);
+      mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); mbar_init(xtma + i, 4);
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 4);
     }
@@ -166,7 +165,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
-  mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
+  // Programmatic dependent launch: the setup above overlaps the previous kernel's
+  // tail; everything below reads what it wrote (block list, counts, queue state).
+  grid_dep_wait();
+  grid_dep_launch_dependents();
+  const uint32_t nblocks = *a.nblocks;
+  const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
+  if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
+  if (warp < cs::GATHER_WARP0) mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
   const float* sb1 = reinterpret_cast<const float*>(sm + cs::BIAS_OFF);
   const float* sb2 = sb1 + 64;
   const float* sb3 = sb1 + 192;
@@ -401,17 +407,21 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (lane == 0) mbar_arrive(stg_empty);
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
-    // Thread m builds rows 2j and 2j+1 of block m for the 4 conv1 positions j of
-    // each tile.  Operand row layout (per input row, 64 bf16): cols 0..46 the
-    // trace attributes (pre-converted once per run into trace16, copied with
-    // cp.async straight into the SWIZZLE_128B tile), col 47 zero, cols 48..50 the
-    // time features (one 16-byte store), cols 51..63 zero (chunk 7 is zeroed
-    // once).  The copies of item n are in flight while item n-1 is signalled:
-    // xfull(n-1) is arrived after cp.async.wait_group<1> + fence.proxy.async.
-    // No load result is consumed in the iteration that issues it: block ids of
-    // tile t+2 are loaded at position 0 of tile t, their sub-trace state at
-    // position 2, queue entries of item n+1 during item n.
+    // Thread m owns block m of each tile and builds its input rows 2j and 2j+1 for
+    // the 4 conv1 positions j (items).  Operand row layout (per input row, 64 bf16):
+    // cols 0..46 the trace attributes, col 47 zero, cols 48..50 the time features,
+    // cols 51..63 zero.  The 128-B rows are fetched by the TMA unit with
+    // tile::gather4 (4 arbitrary trace16 rows per instruction, SWIZZLE_128B applied
+    // on the way): padding rows point at the all-zero row past the rank's rows, the
+    // current instruction at its own row (time features 0), context rows at the row
+    // of their queue entry.  Once an item's rows have landed (xtma), the owner
+    // threads overwrite chunk 6 of their context rows with the time features and
+    // signal xfull.  Two items are in flight: item n is issued before item n-1 is
+    // completed.  No load result is consumed in the iteration that issues it: block
+    // ids of tile t+2 are loaded at position 0 of tile t, their sub-trace state at
+    // position 2, queue entries of item n+2 during item n.
     const int m = tid - cs::GATHER_WARP0 * 32;
+    const int wq = warp - cs::GATHER_WARP0;          // gather warp 0..3: tile rows 32 wq .. 32 wq + 31
     // Every load below is UNCONDITIONAL (out-of-range lanes read a clamped, valid
     // address) and lands in a register of its own: a predicated load merged into a
     // pre-set value would make the merge wait for the load where it is issued.
@@ -434,32 +444,23 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       const int ent = en.kind == 2 ? mt.k - R : 0;        // context newest first (R6)
       en.v = a.q[(uint64_t)ent * a.qn + (mt.id >> 4)];
     };
-    // One input row -> row m of an X atom, owner part: the time features (chunk 6) or,
-    // for a padding row, zeros in chunks 0..6.  Returns the trace16 row offset the
-    // attribute chunks 0..5 are copied from (NONE for padding).
-    constexpr uint32_t NONE = 0xFFFFFFFFu;
-    auto own = [&](const Ent& en, const Meta& mt, uint8_t* atom) -> uint32_t {
-      if (en.kind) {
-        int t0 = 0, t1 = 0, t2 = 0;
-        uint32_t seq = mt.i + (uint32_t)a.step;      // R == 0: current instruction first
-        if (en.kind == 2) {                          // time relative to Clock (R2)
-          const int c = en.v.z & 0xFFFF, sv = en.v.z >> 16;
-          const int age = (int)(mt.clo - en.v.y);
-          t0 = min(age, kTimeMax); t1 = min(max(0, c - age), kTimeMax); t2 = min(c + sv - age, kTimeMax);
-          seq = en.v.x;
-        }
-        st_sw128(atom, m, 6, make_uint4(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f), 0u, 0u));
-        return (uint32_t)((int64_t)seq - a.row_lo);
-      }
-#pragma unroll
-      for (int c = 0; c < 7; ++c) st_sw128(atom, m, c, make_uint4(0, 0, 0, 0));
-      return NONE;
+    // One input row: the trace16 row the TMA fetches, and the time-feature chunk
+    // (cols 48..55) written after it lands (context rows only, R2).
+    auto row_of = [&](const Ent& en, const Meta& mt, uint2& tchunk) -> uint32_t {
+      tchunk = make_uint2(0u, 0u);
+      if (en.kind == 0) return a.zero_row;             // zero padding at the tail
+      if (en.kind == 1) return (uint32_t)((int64_t)(mt.i + (uint32_t)a.step) - a.row_lo);   // current first
+      const int c = en.v.z & 0xFFFF, sv = (en.v.z >> 16) & 0xFFFF;
+      const int age = (int)(mt.clo - en.v.y);
+      const int t0 = min(age, kTimeMax), t1 = min(max(0, c - age), kTimeMax), t2 = min(c + sv - age, kTimeMax);
+      tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
+      return (uint32_t)((int64_t)en.v.x - a.row_lo);
     };
-    // chunk 7 (cols 56..63) of every X row is always zero
+#ifdef PSIM_GATHER_SPLIT
+    // chunk 7 (cols 56..63) of the cp.async rows (atom 1) is never written: zero it once
 #pragma unroll
-    for (int s2 = 0; s2 < 2; ++s2)
-#pragma unroll
-      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
+    for (int s2 = 0; s2 < 2; ++s2) st_sw128(sm + cs::X_OFF + s2 * 32768 + 16384, m, 7, make_uint4(0, 0, 0, 0));
+#endif
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const uint32_t n_items = my_tiles * 4;
     Meta m0, m1, m2;                                  // tiles it, it+1, it+2
@@ -470,6 +471,23 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     Ent ea, eb, ea2, eb2;                             // raw queue parts of items n, n+1
     if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
     if (n_items > 1) { stage_a(m0, 1, 0, ea2); stage_a(m0, 1, 1, eb2); }
+    uint2 pA = make_uint2(0u, 0u), pB = make_uint2(0u, 0u);   // time chunks of item n-1
+    // item n-1 landed -> time features of its context rows -> visible to tcgen05 -> xfull
+    auto complete = [&](uint32_t nprev, bool last) {
+      const int sp = (int)(nprev & 1u);
+      wait_full(xtma + sp, nprev >> 1);
+      uint8_t* xp = sm + cs::X_OFF + sp * 32768;
+      if (pA.x | pA.y) st_sw128(xp, m, 6, make_uint4(pA.x, pA.y, 0u, 0u));
+#ifdef PSIM_GATHER_SPLIT
+      if (last) cp_async_wait<0>(); else cp_async_wait<1>();   // this thread's atom-1 rows of item nprev
+#else
+      (void)last;
+      if (pB.x | pB.y) st_sw128(xp + 16384, m, 6, make_uint4(pB.x, pB.y, 0u, 0u));
+#endif
+      fence_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(xfull + sp);
+    };
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
@@ -478,28 +496,45 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (j == 2) meta_state(m2);
       if (j == 0 && warp == cs::GATHER_WARP0) PSIM_TS(80);
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      uint2 tA, tB;
+      const uint32_t rA = row_of(ea, m0, tA);
+      const uint32_t rB = row_of(eb, m0, tB);
       wait_empty(xempty + s, it * 2 + (j >> 1));
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
       {
         uint8_t* xa = sm + cs::X_OFF + s * 32768;
-        const uint32_t offA = own(ea, m0, xa);
-        if (warp == cs::GATHER_WARP0) PSIM_TS(104 + 2 * j);
-        const uint32_t offB = own(eb, m0, xa + 16384);
-        if (warp == cs::GATHER_WARP0) PSIM_TS(105 + 2 * j);
-        if (offA != NONE) {
+#ifdef PSIM_GATHER_SPLIT
+        // rows 2j (atom 0) by TMA gather4, rows 2j+1 (atom 1) by cp.async: the two copy
+        // engines (TMA unit, LSU) work side by side
+        if (lane == 0) mbar_expect_tx(xtma + s, 32 * 128);   // this warp's 32 atom-0 rows
+        __syncwarp();
+        const int g = lane & 7;
+        uint32_t r4[4];
 #pragma unroll
-          for (int c = 0; c < 6; ++c)
-            cp_async16(xa + m * 128 + ((c ^ (m & 7)) << 4),
-                       reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)offA * 64) + c * 16);
-        }
-        if (offB != NONE) {
+        for (int t = 0; t < 4; ++t) r4[t] = __shfl_sync(0xffffffffu, rA, 4 * g + t);
+        if (lane < 8) tma_gather4(xa + (32 * wq + 4 * g) * 128, &tmX, xtma + s, 0, r4[0], r4[1], r4[2], r4[3]);
+        uint8_t* xb = xa + 16384;
+        const uint8_t* src = reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)rB * 64);
 #pragma unroll
-          for (int c = 0; c < 6; ++c)
-            cp_async16(xa + 16384 + m * 128 + ((c ^ (m & 7)) << 4),
-                       reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)offB * 64) + c * 16);
+        for (int c = 0; c < 6; ++c) cp_async16(xb + m * 128 + ((c ^ (m & 7)) << 4), src + c * 16);
+        cp_async_commit();
+        st_sw128(xb, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));   // time features of row 2j+1 (or zeros)
+#else
+        if (lane == 0) mbar_expect_tx(xtma + s, 64 * 128);   // this warp's 64 rows
+        __syncwarp();
+        // lane l < 16 fetches rows (atom h = l >> 3) of blocks 32 wq + 4 g .. + 3, g = l & 7
+        const int g = lane & 7, h = (lane >> 3) & 1;
+        uint32_t r4[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const uint32_t va = __shfl_sync(0xffffffffu, rA, 4 * g + t);
+          const uint32_t vb = __shfl_sync(0xffffffffu, rB, 4 * g + t);
+          r4[t] = h ? vb : va;
         }
+        if (lane < 16)
+          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xtma + s, 0, r4[0], r4[1], r4[2], r4[3]);
+#endif
       }
-      cp_async_commit();
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
       ea = ea2; eb = eb2;                             // item n+1's raw queue entries
       if (nI + 2 < n_items) {                         // raw queue entries of item n+2
@@ -507,21 +542,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         stage_a(mm, (j + 2) & 3, 0, ea2); stage_a(mm, (j + 2) & 3, 1, eb2);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
-      if (nI > 0) {                                   // item n-1 landed -> visible to tcgen05
-        cp_async_wait<1>();
-        fence_async_smem();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(xfull + ((j + 1) & 1));
-      }
+      if (nI > 0) complete(nI - 1, false);
+      pA = tA; pB = tB;
       if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
       if (j == 3) { m0 = m1; m1 = m2; }               // next tile
     }
-    if (n_items > 0) {                                // the last item
-      cp_async_wait<0>();
-      fence_async_smem();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(xfull + (((n_items - 1) & 3) & 1));
-    }
+    if (n_items > 0) complete(n_items - 1, true);     // the last item
   }
   fence_before();
   __syncthreads();
@@ -607,6 +633,8 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
+  grid_dep_wait();                 // PDL: a4, block counts and queue state of conv_stack / the previous step
+  grid_dep_launch_dependents();
   const bool run_head = (a.u.forced == nullptr) || a.force_predict;
   if (warp >= 2 && warp < 6) mbar_wait(cbar, 0);   // epilogue warps read T and fc2 from smem
 
@@ -959,6 +987,24 @@ static int sm_count() {
   return n;
 }
 
+// launch with programmatic stream serialization (PDL): the kernel may start while the
+// previous kernel on the stream drains; it calls griddepcontrol.wait before touching
+// anything that kernel produced
+template <typename... KArgs, typename... Args>
+static void launch_pdl(void (*kern)(KArgs...), int grid, int threads, int smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3((unsigned)threads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st) {
   const uint64_t th = n > 1 ? n : 1;
   fused_init_kernel<<<(unsigned)((th + 255) / 256), 256, 0, st>>>(n, f.blocks, f.count + 0, f.tileP[0], f.count + 1);
@@ -1001,6 +1047,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   a.nblocks = f.count + (step & 1);
   a.next_count = f.count + ((step + 1) & 1);
   a.trace16 = f.trace16; a.row_lo = g.row_lo;
+  a.zero_row = f.zero_row;
   a.ws = g.ws; a.clock = g.clock; a.count = g.count;
   a.q = g.q;
   a.step = step;
@@ -1013,7 +1060,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   // (n*14 blocks at most); CTAs with no tile exit after setup.
   const uint64_t max_tiles = (n * 14 + cs::TILE - 1) / cs::TILE;
   const int grid = (int)std::min<uint64_t>(max_tiles, (uint64_t)sm_count());
-  conv_stack_kernel<<<grid, cs::THREADS, cs::SMEM, st>>>(a, f.mapW1, f.mapW2, f.mapW3);
+  launch_pdl(conv_stack_kernel, grid, cs::THREADS, cs::SMEM, st, a, f.mapW1, f.mapW2, f.mapW3, f.mapX);
 }
 
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
@@ -1037,12 +1084,17 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
   a.ptile_sum = u.st.ptile_sum;
   const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
   const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
-  fc1_head_kernel<<<grid, fh::THREADS, fh::SMEM, st>>>(f.mapA, f.mapB, a);
+  launch_pdl(fc1_head_kernel, grid, fh::THREADS, fh::SMEM, st, f.mapA, f.mapB, a);
 }
 
 bool fused_make_weight_maps(FusedC3& f) {
   return map2d(&f.mapW1, f.w1p, 64, 128, 64) && map2d(&f.mapW2, f.w2, 128, 128, 128) &&
          map2d(&f.mapW3, f.w3, 128, 256, 128);
+}
+
+bool fused_make_trace_map(FusedC3& f, uint64_t rows) {
+  f.zero_row = (uint32_t)rows;
+  return map2d(&f.mapX, f.trace16, rows + 1, 64, 1);
 }
 
 bool fused_make_maps(FusedC3& f, uint64_t n) {

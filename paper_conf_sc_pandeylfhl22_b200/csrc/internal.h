@@ -196,6 +196,8 @@ struct FusedC3 {
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
   CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
+  CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][64] (box 64 x 1, SWIZZLE_128B)
+  uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)
 };
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
 // block list / P_tile of step 0 of a pass whose sub-traces start from a non-empty
@@ -214,6 +216,8 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
                      cudaStream_t st);
 bool fused_make_maps(FusedC3& f, uint64_t n);
 bool fused_make_weight_maps(FusedC3& f);
+// gather4 map of f.trace16 with rows + 1 rows (the last one zero); sets f.zero_row
+bool fused_make_trace_map(FusedC3& f, uint64_t rows);
 void fused_dump_debug();
 
 // pad/convert the caller's [B][112][50] fp32 inputs (psim_cnn_forward)

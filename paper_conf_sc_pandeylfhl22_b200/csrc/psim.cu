@@ -63,6 +63,10 @@ inline uint16_t f32_to_bf16_rne(float f) {
 // (PSIM_PROFILE); launch counting is always on (psim_stats.gpu_launches).
 struct Prof {
   bool on = false;
+  bool sample = true;          // time this launch (lockstep kernels: every kEvery-th step only,
+                               // so the events do not serialise the PDL overlap of the others)
+  static constexpr int kEvery = 16;
+  uint64_t timed[PSIM_KC_COUNT] = {};
   cudaStream_t st = nullptr;
   std::vector<cudaEvent_t> pool;
   size_t used = 0;
@@ -70,8 +74,9 @@ struct Prof {
   size_t open_idx = 0;
   uint64_t launches[PSIM_KC_COUNT] = {};
   void reset(bool enable, cudaStream_t s) {
-    on = enable; st = s; used = 0; marks.clear();
+    on = enable; st = s; used = 0; marks.clear(); sample = true;
     for (auto& l : launches) l = 0;
+    for (auto& l : timed) l = 0;
   }
   cudaEvent_t next() {
     if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
@@ -79,15 +84,17 @@ struct Prof {
   }
   void begin(int cls) {
     launches[cls]++;
-    if (!on) return;
+    if (!on || !sample) return;
+    timed[cls]++;
     open_idx = used;
     cudaEventRecord(next(), st);
   }
   void end(int cls) {
-    if (!on) return;
+    if (!on || !sample) return;
     cudaEventRecord(next(), st);
     marks.push_back({cls, open_idx});
   }
+  // per-class device time, scaled from the timed launches to all launches of the class
   void collect(double* ms) {
     for (int c = 0; c < PSIM_KC_COUNT; ++c) ms[c] = 0;
     for (auto& m : marks) {
@@ -95,6 +102,8 @@ struct Prof {
       cudaEventElapsedTime(&t, pool[m.second], pool[m.second + 1]);
       ms[m.first] += t;
     }
+    for (int c = 0; c < PSIM_KC_COUNT; ++c)
+      if (timed[c]) ms[c] *= (double)launches[c] / (double)timed[c];
   }
   ~Prof() { for (auto e : pool) cudaEventDestroy(e); }
 };
@@ -812,6 +821,10 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       CK(cudaMalloc(&ctx->fused.trace16, t16 + 256));
       ctx->fused.trace16_cap = t16;
     }
+    // row `rows` of trace16 is all zero: the padding rows of the gathered input point at it
+    CK(cudaMemsetAsync(ctx->fused.trace16 + (size_t)rows * 64, 0, 128, st));
+    if (!fused_make_trace_map(ctx->fused, (uint64_t)rows))
+      FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for the trace gather map");
     if (stream_load) {
       if (!ctx->ld_stream) CK(cudaStreamCreateWithFlags(&ctx->ld_stream, cudaStreamNonBlocking));
       const size_t nch = (size_t)((ctx->steps + chunk - 1) / chunk);
@@ -869,9 +882,11 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   };
   for (int64_t t = 0; t < ctx->steps && n; ++t) {
     if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
+    pf.sample = t % Prof::kEvery == 0;
     rc = step(ga, ua, ctx->st.e, t);
     if (rc) return rc;
   }
+  pf.sample = true;
   // ---- post-error correction pass (PAPER.md:203-219 [V-B], Fig. 9; R19) ----
   // corrector b continues from its final state over rows of sub-trace b+1 (same
   // kernels, lockstep over correctors, at most `limit` steps), then the
@@ -906,9 +921,11 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       pf.end(PSIM_KC_OTHER);
     }
     for (int64_t t = 0; t < p.limit; ++t) {
+      pf.sample = t % Prof::kEvery == 0;
       rc = step(g2, u2, p.e, t);
       if (rc) return rc;
     }
+    pf.sample = true;
     pf.begin(PSIM_KC_OTHER);
     launch_pec_apply(ctx->st, p, st);
     pf.end(PSIM_KC_OTHER);

@@ -45,6 +45,30 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       : "memory");
 }
 // 1-D bulk copy global -> shared (size multiple of 16, both 16-byte aligned)
+// TMA tile::gather4 (sm_100): rows r0..r3 (columns c0 .. c0 + box cols) of a 2-D tensor
+// map with box rows = 1 into 4 consecutive 128-B smem rows at dst, swizzled as the
+// map says (SWIZZLE_128B lands in the K-major SW128 operand layout at any 512-B offset)
+__device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, uint32_t r0,
+                                            uint32_t r1, uint32_t r2, uint32_t r3) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, "
+      "%5, %6}], [%7];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar))
+      : "memory");
+}
+// L2 prefetch of 4 rows of a gather4 map (no smem, no barrier)
+__device__ __forceinline__ void tma_prefetch_gather4(const CUtensorMap* map, int c0, uint32_t r0, uint32_t r1,
+                                                     uint32_t r2, uint32_t r3) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile::gather4 [%0, {%1, %2, %3, %4, %5}];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3)
+               : "memory");
+}
+// programmatic dependent launch (PDL)
+__device__ __forceinline__ void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void grid_dep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                    smem_u32(dst)),
