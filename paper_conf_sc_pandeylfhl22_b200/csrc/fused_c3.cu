@@ -700,11 +700,14 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         fence_after();
         y0 = sW2[768]; y1 = sW2[769]; y2 = sW2[770];
         const float* Trow = sT + pb * fh::T_STRIDE;
-        // fc1 = F (positions < P_tile; rows [P_b, P_tile) are zero) + T[P_b]; ReLU; fc2 (R16, R18)
-#pragma unroll 1
-        for (int cc = 0; cc < fh::BN / 32; ++cc) {
-          uint32_t r0[32];
-          tmem_ld32(tmem + lane_base + acc * fh::BN + cc * 32, r0);
+        // fc1 = F (positions < P_tile; rows [P_b, P_tile) are zero) + T[P_b]; ReLU; fc2 (R16, R18).
+        // Two TMEM loads in flight (the next 32 columns load while these are consumed) and
+        // two partial sums per output (halves the dependent FMA chains).
+        float z0 = 0.f, z1 = 0.f, z2 = 0.f;
+        const uint32_t tbase = tmem + lane_base + acc * fh::BN;
+        uint32_t ra[32], rb[32];
+        tmem_ld32_nowait(tbase, ra);
+        auto consume = [&](const uint32_t (&r0)[32], int cc) {
 #pragma unroll
           for (int j4 = 0; j4 < 8; ++j4) {
             const int col = cc * 32 + j4 * 4;
@@ -716,11 +719,21 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
             const float f2 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 2]) : 0.f, f3 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 3]) : 0.f;
             const float h0 = fmaxf(f0 + tv.x, 0.f), h1 = fmaxf(f1 + tv.y, 0.f);
             const float h2 = fmaxf(f2 + tv.z, 0.f), h3 = fmaxf(f3 + tv.w, 0.f);
-            y0 = fmaf(h0, w0.x, y0); y0 = fmaf(h1, w0.y, y0); y0 = fmaf(h2, w0.z, y0); y0 = fmaf(h3, w0.w, y0);
-            y1 = fmaf(h0, w1.x, y1); y1 = fmaf(h1, w1.y, y1); y1 = fmaf(h2, w1.z, y1); y1 = fmaf(h3, w1.w, y1);
-            y2 = fmaf(h0, w2v.x, y2); y2 = fmaf(h1, w2v.y, y2); y2 = fmaf(h2, w2v.z, y2); y2 = fmaf(h3, w2v.w, y2);
+            y0 = fmaf(h0, w0.x, y0); z0 = fmaf(h1, w0.y, z0); y0 = fmaf(h2, w0.z, y0); z0 = fmaf(h3, w0.w, z0);
+            y1 = fmaf(h0, w1.x, y1); z1 = fmaf(h1, w1.y, z1); y1 = fmaf(h2, w1.z, y1); z1 = fmaf(h3, w1.w, z1);
+            y2 = fmaf(h0, w2v.x, y2); z2 = fmaf(h1, w2v.y, z2); y2 = fmaf(h2, w2v.z, y2); z2 = fmaf(h3, w2v.w, z2);
           }
+        };
+#pragma unroll 1
+        for (int cc = 0; cc < fh::BN / 32; cc += 2) {
+          tmem_wait_ld();                                   // columns cc (ra) landed
+          tmem_ld32_nowait(tbase + (cc + 1) * 32, rb);
+          consume(ra, cc);
+          tmem_wait_ld();                                   // columns cc + 1 (rb) landed
+          if (cc + 2 < fh::BN / 32) tmem_ld32_nowait(tbase + (cc + 2) * 32, ra);
+          consume(rb, cc + 1);
         }
+        y0 += z0; y1 += z1; y2 += z2;
         fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(tempty + acc);
@@ -746,9 +759,10 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const int tileP_cur = a.tileP[tt];
       int64_t ws = 0, s_b = 0, nsteps = 0, clock = 0;
       int kb = 0;
+      uint32_t rmin = 0;
       if (inb) {   // prefetch the state and the first queue entries while the head runs
         ws = a.u.st.ws[b]; s_b = a.u.st.s[b]; nsteps = a.e[b] - ws;
-        kb = a.u.st.count[b]; clock = a.u.st.clock[b];
+        kb = a.u.st.count[b]; clock = a.u.st.clock[b]; rmin = a.u.st.rmin[b];
       }
       const bool active = inb && a.u.step < nsteps;
       QBatch first;
@@ -763,7 +777,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       int pnext = 0;
       if (active) {
         bool stopped = false;
-        const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, first, run_head, y0, y1, y2, sHist,
+        const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, rmin, first, run_head, y0, y1, y2, sHist,
                                                 &stopped);
         if (a.u.step + 1 < nsteps && !stopped) {
           pnext = (knew + 8) >> 3;                 // ceil((k+1)/8)

@@ -61,6 +61,8 @@ struct SimState {
   int64_t* bnd = nullptr;       // [n] Clock at the end of warm-up
   int64_t* cycles = nullptr;    // [n] Clock_end - bnd
   int32_t* count = nullptr;     // [n] live context entries
+  uint32_t* rmin = nullptr;     // [n] low 32 bits of the smallest retire Clock of the live entries
+                                // (valid when count > 0; maintained by the thread-per-sub-trace update)
   // queue entries are ENTRY-MAJOR: entry e of sub-trace b at [e * n + b], so the
   // threads of a warp (consecutive sub-traces) touch consecutive 16-byte words, and
   // one entry is one 16-byte load (one DRAM sector) for the gather

@@ -235,7 +235,7 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->model.head_b);
   SimState& s = ctx->st;
   for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
-                  (void*)s.count, (void*)s.q, (void*)s.k_hist,
+                  (void*)s.count, (void*)s.q, (void*)s.rmin, (void*)s.k_hist,
                   (void*)s.stalls, (void*)s.total, (void*)s.ptile_sum})
     dfree(p);
   dfree(ctx->buf.x);
@@ -633,9 +633,10 @@ static int ensure_state(psim_ctx* ctx) {
   SimState& s = ctx->st;
   if (ctx->st_cap < n || !s.clock) {
     for (void* p : {(void*)s.ws, (void*)s.s, (void*)s.e, (void*)s.clock, (void*)s.bnd, (void*)s.cycles,
-                    (void*)s.count, (void*)s.q})
+                    (void*)s.count, (void*)s.q, (void*)s.rmin})
       dfree(p);
     const uint64_t a = std::max<uint64_t>(n, 1);
+    CK(cudaMalloc(&s.rmin, a * 4));
     CK(cudaMalloc(&s.ws, a * 8)); CK(cudaMalloc(&s.s, a * 8)); CK(cudaMalloc(&s.e, a * 8));
     CK(cudaMalloc(&s.clock, a * 8)); CK(cudaMalloc(&s.bnd, a * 8)); CK(cudaMalloc(&s.cycles, a * 8));
     CK(cudaMalloc(&s.count, a * 4));

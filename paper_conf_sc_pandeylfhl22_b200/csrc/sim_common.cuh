@@ -186,8 +186,8 @@ __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int 
 }
 
 __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
-                                                      int64_t nsteps, int k, int64_t clock, const QBatch& first,
-                                                      bool has_y, float y0, float y1, float y2,
+                                                      int64_t nsteps, int k, int64_t clock, uint32_t rmin,
+                                                      const QBatch& first, bool has_y, float y0, float y1, float y2,
                                                       unsigned int* hist, bool* stopped = nullptr) {
   const int64_t i = ws + a.step;
   int f, c, s;
@@ -214,6 +214,20 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
   const int n_in = k + 1;
   int w = 0, nst = 0;
   int dmin = 0x7fffffff;   // min (retire - Clock) over kept entries
+  const bool new_live = (c + s) > 0;                       // retire = Clock + c + s > Clock
+  // Fast path: if the smallest retire Clock of the old entries is still ahead of the new
+  // Clock, none of them retires; only the pushed entry is appended (or retires at once).
+  // The result is the same set removal as the scan below.
+  if (k == 0 || (int)(rmin - clo) > 0) {
+    if (k + (new_live ? 1 : 0) <= a.cap) {
+      if (new_live) qb[(uint64_t)k * qn] = make_uint4(push_s, push_f, push_c, push_w);
+      w = k + (new_live ? 1 : 0);
+      nst = new_live ? 0 : (int)(push_w & 1u);
+      const uint32_t rnew = clo + (uint32_t)(c + s);
+      rmin = (k == 0 || (int)(rnew - rmin) < 0) ? rnew : rmin;
+      goto done;
+    }
+  }
   for (int e0 = 0; e0 < n_in; e0 += 8) {
     uint32_t vs[8], vf[8], vc[8], vw[8];
 #pragma unroll
@@ -242,18 +256,24 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
     clo = (uint32_t)clock;
     const int n2 = w;
     w = 0;
+    dmin = 0x7fffffff;
     for (int e = 0; e < n2; ++e) {
       const uint4 v = qb[e * qn];
-      if ((int)(v.z & 0xFFFF) + (int)(v.z >> 16) - (int)(clo - v.y) > 0) {
+      const int rem = (int)(v.z & 0xFFFF) + (int)(v.z >> 16) - (int)(clo - v.y);
+      if (rem > 0) {
         qb[w * qn] = v; ++w;
+        dmin = min(dmin, rem);
       } else {
         nst += (int)(v.w & 1u);
       }
     }
     atomicAdd(a.st.stalls, 1ull);
   }
+  rmin = clo + (uint32_t)dmin;                             // (unused when w == 0)
+done:
   a.st.count[b] = w;
   a.st.clock[b] = clock;
+  a.st.rmin[b] = rmin;
   int64_t bnd = a.st.bnd[b];
   if (i == s_b - 1) { bnd = clock; a.st.bnd[b] = bnd; }   // end of warm-up
   if (a.step == nsteps - 1) a.st.cycles[b] = clock - bnd;

@@ -56,6 +56,12 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, u
       "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar))
       : "memory");
 }
+// L2 prefetch of one box of a 2-D tensor map (no smem, no barrier)
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, int c1) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
 // L2 prefetch of 4 rows of a gather4 map (no smem, no barrier)
 __device__ __forceinline__ void tma_prefetch_gather4(const CUtensorMap* map, int c0, uint32_t r0, uint32_t r1,
                                                      uint32_t r2, uint32_t r3) {
