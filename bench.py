@@ -218,6 +218,9 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg (profiling runs)")
+    ap.add_argument("--emulate-rank", default=None, metavar="R/G",
+                    help="diagnostics: run rank R's share of a G-GPU job on this one GPU (no NCCL), "
+                         "to estimate per-GPU throughput at G GPUs; value = that rank's instructions/s")
     ap.add_argument("--correction", type=int, default=0,
                     help="post-error correction limit (PAPER.md:203-219; the paper uses 100); 0 = off")
     args = ap.parse_args()
@@ -226,6 +229,9 @@ def main():
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    emu = None
+    if args.emulate_rank:
+        emu = tuple(int(x) for x in args.emulate_rank.split("/"))   # (R, G): partition as rank R of G
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     config = {"workload": cfg["desc"], "instructions": L, "subtraces": N, "warmup_W": W, "cnn": cfg["arch"],
               "queue_rows": 111, "precision": cfg["precision"],
@@ -271,7 +277,7 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
 
-    rr = P.partition_range(L, N, W, rank, world)
+    rr = P.partition_range(L, N, W, *(emu if emu else (rank, world)))
     rows = rr.row_hi - rr.row_lo
     t0 = time.time()
     host = torch.empty((rows, 48), dtype=torch.uint8, pin_memory=True)
@@ -294,7 +300,8 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=rank, world_size=world, nccl_id=nccl_id,
+    sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=emu[0] if emu else rank,
+                      world_size=emu[1] if emu else world, nccl_id=nccl_id,
                       stream=stream.cuda_stream, profile=os.environ.get("PSIM_NOPROF") is None, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")),
                       correction_limit=args.correction)
     sim.load_model(cfg["arch"], w)
@@ -324,6 +331,9 @@ def main():
 
     ms, total, stats, clocks = timed(dev, args.steps, args.warmup)
     value = L * args.steps / (ms / 1e3) / 1e6
+    if emu:   # this rank's counted instructions only
+        value = stats["counted"] * args.steps / (ms / 1e3) / 1e6
+        config["emulated_rank"] = f"{emu[0]}/{emu[1]} (one GPU's share of a {emu[1]}-GPU job, no NCCL)"
     e2e = None
     if not args.no_e2e:
         ms_e, total_e, st_e, _ = timed(host, args.steps, 1)

@@ -44,23 +44,26 @@ constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
 constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
 constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of W3, streamed by TMA
                                              // (halves alternate with the conv3 MMAs, from L2)
-constexpr int X_OFF = W3_OFF + 32 * 1024;    // 2 slots x 2 atoms [128][64]
-constexpr int A2_OFF = X_OFF + 64 * 1024;    // 1 atom  [128][64]
+constexpr int NX = 3;                        // X slots: gathered items in flight
+constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
+constexpr int A2_OFF = X_OFF + NX * 32 * 1024;   // 1 atom  [128][64]
 constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
-constexpr int STG_OFF = A3_OFF + 32 * 1024;  // 128 staged conv3 rows (256 B each) for the write-back warp
-constexpr int BAR_OFF = STG_OFF + 32 * 1024; // mbarriers
-constexpr int BIAS_OFF = BAR_OFF + 256;      // b1[64] b2[128] b3[128] fp32
+constexpr int BAR_OFF = A3_OFF + 32 * 1024;  // mbarriers
+constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
-constexpr int THREADS = 448;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi), 8 MMA, 9-12 gather, 13 write-back
-constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, WB_WARP = 13;
+constexpr int THREADS = 416;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 gather
+constexpr int MMA_WARP = 8, GATHER_WARP0 = 9;
+#ifndef PSIM_GATHER_DEPTH
+#define PSIM_GATHER_DEPTH 1        // items issued ahead of the one being completed
+#endif
 }  // namespace cs
 
 struct ConvArgs {
   const uint32_t* blocks;    // block ids (b << 4 | p) of this step
   const uint32_t* nblocks;   // count of this step's list
   uint32_t* next_count;      // the other step parity's counter, reset here
-  const __nv_bfloat16* trace16;   // [rows + 1][64] bf16 operand rows (attributes at cols 0..46), row `rows` zero
+  const __nv_bfloat16* trace16;   // [rows + 1][48] bf16 operand rows (attributes at cols 0..46), row `rows` zero
   uint32_t zero_row;         // index of the all-zero trace16 row (padding rows of the input)
   int64_t row_lo;
   const int64_t* ws;
@@ -117,8 +120,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
-  uint64_t* xfull = bars + 0;      // [2] 4 gather warps
-  uint64_t* xempty = bars + 2;     // [2] commit
+  uint64_t* xfull = bars + 24;     // [NX] 4 gather warps
+  uint64_t* xempty = bars + 28;    // [NX] commit
   uint64_t* c1full = bars + 4;     // [2] commit
   uint64_t* c1empty = bars + 6;    // [2] 4 (EG-A)
   uint64_t* a2full = bars + 8;     //     4 (EG-A)
@@ -130,25 +133,22 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* c3full = bars + 16;    //     commit
   uint64_t* c3empty = bars + 17;   //     4 (EG-B)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
-  uint64_t* stg_full = bars + 19;  //     4 (EG-B): conv3 rows staged in STG
-  uint64_t* stg_empty = bars + 20; //     1 (write-back warp)
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
-  uint64_t* xtma = bars + 23;      // [2] 4 gather warps (expect_tx) + the gathered rows (complete_tx)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 25);
+  uint64_t* xtma = bars + 32;      // [NX] 4 gather warps (expect_tx) + the gathered rows (complete_tx)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 36);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (tid == 0) {
+    for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); mbar_init(xtma + i, 4); }
     for (int i = 0; i < 2; ++i) {
-      mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); mbar_init(xtma + i, 4);
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 4);
     }
     mbar_init(a2full, 4); mbar_init(a2empty, 1);
     mbar_init(a3full, 4); mbar_init(a3empty, 1); mbar_init(c3full, 1); mbar_init(c3empty, 4);
     mbar_init(wbar, 1);
-    mbar_init(stg_full, 4); mbar_init(stg_empty, 1);
     mbar_init(w3full, 1); mbar_init(w3empty, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     // resident weights W1/W2 (48 KB) by TMA, already in the SWIZZLE_128B operand layout
@@ -184,19 +184,20 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       const uint32_t sbase = smem_u32(sm);
       const uint32_t id64 = idesc_bf16(128, 64), id128 = idesc_bf16(128, 128);
       auto c1 = [&](uint32_t it, int j) {
-        const int s = j & 1;
+        const int s = j & 1;                        // C1 TMEM slot
         const uint32_t n = it * 2 + (j >> 1);
+        const uint32_t item = it * 4 + j, xs = item % cs::NX;   // X slot of this item
         PSIM_TS(0 + 2 * j);
-        wait_full(xfull + s, n);
+        wait_full(xfull + xs, item / cs::NX);
         wait_empty(c1empty + s, n);
         PSIM_TS(1 + 2 * j);
         fence_after();
-        const uint32_t xa = sbase + cs::X_OFF + s * 32768;
+        const uint32_t xa = sbase + cs::X_OFF + xs * 32768;
 #pragma unroll
         for (int k = 0; k < 8; ++k)
           mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
                    sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
-        mma_commit(xempty + s);
+        mma_commit(xempty + xs);
         mma_commit(c1full + s);
       };
       auto c2 = [&](uint32_t it, int h, int kh) {
@@ -318,93 +319,37 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         if (lane == 0) { mbar_arrive(c2empty + h); mbar_arrive(a3full); }
         if (q == 0) PSIM_TS(59 + 4 * h);
       }
-      // C3 (128 fp32) -> relu(+b3) -> bf16 -> plain staging rows in the A3 region -> write-back warp
+      // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p] (256-B row per thread, straight from
+      // registers; the TMA unit stays free for the row gathers)
+      const uint32_t bi = tl * cs::TILE + m;
+      const uint32_t id = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
       wait_full(c3full, it);                          // conv3 accumulated
-      wait_empty(stg_empty, it);                      // previous tile's staging rows written back
       if (q == 0) PSIM_TS(65);
       fence_after();
-      uint8_t* row = sm + cs::STG_OFF + m * 256;
-#pragma unroll 1
-      for (int cp = 0; cp < 2; ++cp) {
+      uint32_t pk[64];
+      {
         uint32_t r0[32], r1[32];
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + cp * 64 + 32, r1);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 32, r1);
         tmem_wait_ld();
-        uint32_t pk[32];
-        bias_relu_pack32(r0, sb3 + cp * 64, pk);
-        bias_relu_pack32(r1, sb3 + cp * 64 + 32, pk + 16);
-        // lane-rotated chunk order (conflict-free stores at a 256-B row pitch): rotate the
-        // 8 chunks left by m & 7 in three conditional stages, then chunk c goes to (c + m) & 7
-        const int r = m & 7;
-#pragma unroll
-        for (int st = 1; st < 8; st <<= 1) {
-          const bool sw = (r & st) != 0;
-          uint32_t t[32];
-#pragma unroll
-          for (int c = 0; c < 32; ++c) t[c] = sw ? pk[(c + 4 * st) & 31] : pk[c];
-#pragma unroll
-          for (int c = 0; c < 32; ++c) pk[c] = t[c];
-        }
-#pragma unroll
-        for (int c = 0; c < 8; ++c)
-          *reinterpret_cast<uint4*>(row + (cp * 8 + ((c + r) & 7)) * 16) =
-              make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+        bias_relu_pack32(r0, sb3, pk);
+        bias_relu_pack32(r1, sb3 + 32, pk + 16);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 64, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 96, r1);
+        tmem_wait_ld();
+        bias_relu_pack32(r0, sb3 + 64, pk + 32);
+        bias_relu_pack32(r1, sb3 + 96, pk + 48);
       }
       fence_before();
-      fence_async_smem();                             // staging rows are read by TMA bulk copies
       __syncwarp();
-      if (lane == 0) { mbar_arrive(c3empty); mbar_arrive(stg_full); }
+      if (lane == 0) mbar_arrive(c3empty);            // C3 TMEM free for the next tile's conv3
+      if (id != 0xFFFFFFFFu) {
+        uint4* dst = reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128);
+#pragma unroll
+        for (int c = 0; c < 16; ++c) dst[c] = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+      }
       if (q == 0) PSIM_TS(66);
-    }
-  } else if (warp == cs::WB_WARP) {   // ============================ a4 write-back
-    // the 128 staged conv3 rows (256 B each) of a tile -> a4[b][p] by TMA bulk stores,
-    // off the epilogues' critical path
-    // Block ids are b-major with consecutive positions, so the rows of one sub-trace
-    // form a contiguous run in the staging area AND in a4[b][p..]: one bulk copy per
-    // run (mean ~3 rows) instead of one per row -- the TMA unit's per-copy cost was
-    // on the critical path (A3 is reused by the next tile's conv2 epilogue).
-    // Lane l owns tile rows 4l..4l+3; the next 16 rows come from lanes l+1..l+4.
-    constexpr uint32_t NONE = 0xFFFFFFFFu;
-    uint32_t it = 0;
-    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
-      uint32_t ids[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const uint32_t bi = tl * cs::TILE + 4 * lane + u;
-        ids[u] = bi < nblocks ? a.blocks[bi] : NONE;
-      }
-      uint32_t nxt[16];
-#pragma unroll
-      for (int d = 1; d <= 4; ++d)
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const uint32_t v = __shfl_down_sync(0xffffffffu, ids[u], d);
-          nxt[(d - 1) * 4 + u] = lane + d < 32 ? v : NONE;
-        }
-      uint32_t prev = __shfl_up_sync(0xffffffffu, ids[3], 1);
-      if (lane == 0) prev = NONE;
-      wait_full(stg_full, it);
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const uint32_t id = ids[u];
-        const uint32_t before = u == 0 ? prev : ids[u - 1];
-        if (id == NONE || (before != NONE && (before >> 4) == (id >> 4))) continue;   // not a run start
-        int len = 1;
-        bool run = true;
-#pragma unroll
-        for (int v = u + 1; v < u + 14; ++v) {
-          const uint32_t x = v < 4 ? ids[v] : nxt[v - 4];
-          run = run && x != NONE && (x >> 4) == (id >> 4);
-          len += run ? 1 : 0;
-        }
-        bulk_s2g(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128, sm + cs::STG_OFF + (4 * lane + u) * 256,
-                 (uint32_t)len * 256);
-      }
-      bulk_commit();
-      bulk_wait_read();                             // staging rows consumed -> STG reusable
-      __syncwarp();
-      if (lane == 0) mbar_arrive(stg_empty);
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
     // Thread m owns block m of each tile and builds its input rows 2j and 2j+1 for
@@ -456,11 +401,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
       return (uint32_t)((int64_t)en.v.x - a.row_lo);
     };
-#ifdef PSIM_GATHER_SPLIT
-    // chunk 7 (cols 56..63) of the cp.async rows (atom 1) is never written: zero it once
+    // chunk 7 (cols 56..63) of every X row is never written by the TMA: zero it once
 #pragma unroll
-    for (int s2 = 0; s2 < 2; ++s2) st_sw128(sm + cs::X_OFF + s2 * 32768 + 16384, m, 7, make_uint4(0, 0, 0, 0));
-#endif
+    for (int s2 = 0; s2 < cs::NX; ++s2)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const uint32_t n_items = my_tiles * 4;
     Meta m0, m1, m2;                                  // tiles it, it+1, it+2
@@ -471,19 +416,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     Ent ea, eb, ea2, eb2;                             // raw queue parts of items n, n+1
     if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
     if (n_items > 1) { stage_a(m0, 1, 0, ea2); stage_a(m0, 1, 1, eb2); }
-    uint2 pA = make_uint2(0u, 0u), pB = make_uint2(0u, 0u);   // time chunks of item n-1
+    // time chunks of the items issued but not completed yet (n-1, n-2)
+    uint2 pA1 = make_uint2(0u, 0u), pB1 = make_uint2(0u, 0u), pA2 = pA1, pB2 = pA1;
     // item n-1 landed -> time features of its context rows -> visible to tcgen05 -> xfull
-    auto complete = [&](uint32_t nprev, bool last) {
-      const int sp = (int)(nprev & 1u);
-      wait_full(xtma + sp, nprev >> 1);
+    auto complete = [&](uint32_t nprev, uint2 pA, uint2 pB) {
+      const int sp = (int)(nprev % cs::NX);
+      wait_full(xtma + sp, nprev / cs::NX);
       uint8_t* xp = sm + cs::X_OFF + sp * 32768;
-      if (pA.x | pA.y) st_sw128(xp, m, 6, make_uint4(pA.x, pA.y, 0u, 0u));
-#ifdef PSIM_GATHER_SPLIT
-      if (last) cp_async_wait<0>(); else cp_async_wait<1>();   // this thread's atom-1 rows of item nprev
-#else
-      (void)last;
-      if (pB.x | pB.y) st_sw128(xp + 16384, m, 6, make_uint4(pB.x, pB.y, 0u, 0u));
-#endif
+      (void)xp; (void)pA; (void)pB;
       fence_async_smem();
       __syncwarp();
       if (lane == 0) mbar_arrive(xfull + sp);
@@ -499,28 +439,16 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       uint2 tA, tB;
       const uint32_t rA = row_of(ea, m0, tA);
       const uint32_t rB = row_of(eb, m0, tB);
-      wait_empty(xempty + s, it * 2 + (j >> 1));
+      const int xs = (int)(nI % cs::NX);
+      wait_empty(xempty + xs, nI / cs::NX);
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
       {
-        uint8_t* xa = sm + cs::X_OFF + s * 32768;
-#ifdef PSIM_GATHER_SPLIT
-        // rows 2j (atom 0) by TMA gather4, rows 2j+1 (atom 1) by cp.async: the two copy
-        // engines (TMA unit, LSU) work side by side
-        if (lane == 0) mbar_expect_tx(xtma + s, 32 * 128);   // this warp's 32 atom-0 rows
-        __syncwarp();
-        const int g = lane & 7;
-        uint32_t r4[4];
-#pragma unroll
-        for (int t = 0; t < 4; ++t) r4[t] = __shfl_sync(0xffffffffu, rA, 4 * g + t);
-        if (lane < 8) tma_gather4(xa + (32 * wq + 4 * g) * 128, &tmX, xtma + s, 0, r4[0], r4[1], r4[2], r4[3]);
-        uint8_t* xb = xa + 16384;
-        const uint8_t* src = reinterpret_cast<const uint8_t*>(a.trace16 + (uint64_t)rB * 64);
-#pragma unroll
-        for (int c = 0; c < 6; ++c) cp_async16(xb + m * 128 + ((c ^ (m & 7)) << 4), src + c * 16);
-        cp_async_commit();
-        st_sw128(xb, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));   // time features of row 2j+1 (or zeros)
-#else
-        if (lane == 0) mbar_expect_tx(xtma + s, 64 * 128);   // this warp's 64 rows
+        uint8_t* xa = sm + cs::X_OFF + xs * 32768;
+        // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
+        // writes only chunks 0..5, so this can go in before the rows land
+        st_sw128(xa, m, 6, make_uint4(tA.x, tA.y, 0u, 0u));
+        st_sw128(xa + 16384, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));
+        if (lane == 0) mbar_expect_tx(xtma + xs, 64 * 96);    // this warp's 64 rows, 96 B each
         __syncwarp();
         // lane l < 16 fetches rows (atom h = l >> 3) of blocks 32 wq + 4 g .. + 3, g = l & 7
         const int g = lane & 7, h = (lane >> 3) & 1;
@@ -532,8 +460,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           r4[t] = h ? vb : va;
         }
         if (lane < 16)
-          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xtma + s, 0, r4[0], r4[1], r4[2], r4[3]);
-#endif
+          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xtma + xs, 0, r4[0], r4[1], r4[2], r4[3]);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
       ea = ea2; eb = eb2;                             // item n+1's raw queue entries
@@ -542,12 +469,20 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         stage_a(mm, (j + 2) & 3, 0, ea2); stage_a(mm, (j + 2) & 3, 1, eb2);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
-      if (nI > 0) complete(nI - 1, false);
-      pA = tA; pB = tB;
+#if PSIM_GATHER_DEPTH == 2
+      if (nI > 1) complete(nI - 2, pA2, pB2);       // item n-2 landed long ago
+      pA2 = pA1; pB2 = pB1;
+#else
+      if (nI > 0) complete(nI - 1, pA1, pB1);
+#endif
+      pA1 = tA; pB1 = tB;
       if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
       if (j == 3) { m0 = m1; m1 = m2; }               // next tile
     }
-    if (n_items > 0) complete(n_items - 1, true);     // the last item
+#if PSIM_GATHER_DEPTH == 2
+    if (n_items > 1) complete(n_items - 2, pA2, pB2);
+#endif
+    if (n_items > 0) complete(n_items - 1, pA1, pB1);   // the last item
   }
   fence_before();
   __syncthreads();
@@ -833,10 +768,10 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
 // cols 47..63 = 0 (time features are inserted by the gather at cols 48..50)
 __global__ void trace16_kernel(const uint8_t* __restrict__ trace, int64_t stride, int64_t rows,
                                __nv_bfloat16* __restrict__ out) {
-  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;   // one 16-B output chunk
-  if (t >= rows * 8) return;
-  const int64_t r = t >> 3;
-  const int c = (int)(t & 7);
+  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;   // one 16-B output chunk (6 per row)
+  if (t >= rows * 6) return;
+  const int64_t r = t / 6;
+  const int c = (int)(t - r * 6);
   const uint8_t* src = trace + r * stride;
   uint32_t w[4];
 #pragma unroll
@@ -849,7 +784,7 @@ __global__ void trace16_kernel(const uint8_t* __restrict__ trace, int64_t stride
   reinterpret_cast<uint4*>(out)[t] = make_uint4(w[0], w[1], w[2], w[3]);
 }
 void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st) {
-  const int64_t n = rows * 8;
+  const int64_t n = rows * 6;
   if (n > 0) trace16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(trace, stride, rows, out);
 }
 
@@ -896,10 +831,9 @@ __global__ void __launch_bounds__(128) load_chunk16_kernel(const uint8_t* __rest
           const float f1 = a1 < 47 ? (float)((wv[(2 * t + 1) >> 2] >> (((2 * t + 1) & 3) * 8)) & 0xFFu) : 0.f;
           o[t] = pack_bf16(f0, f1);
         }
-        uint4* dst = reinterpret_cast<uint4*>(out + (r - row_lo) * 64);
+        uint4* dst = reinterpret_cast<uint4*>(out + (r - row_lo) * 48);
         dst[2 * q] = make_uint4(o[0], o[1], o[2], o[3]);
         dst[2 * q + 1] = make_uint4(o[4], o[5], o[6], o[7]);
-        if (q == 2) { dst[6] = make_uint4(0, 0, 0, 0); dst[7] = make_uint4(0, 0, 0, 0); }
       }
     }
   }
@@ -1108,7 +1042,16 @@ bool fused_make_weight_maps(FusedC3& f) {
 
 bool fused_make_trace_map(FusedC3& f, uint64_t rows) {
   f.zero_row = (uint32_t)rows;
-  return map2d(&f.mapX, f.trace16, rows + 1, 64, 1);
+  // 96-B rows (48 bf16: 47 attributes + 0); a 48-column box lands in chunks 0..5 of the
+  // 128-B SWIZZLE_128B operand rows, chunks 6 (time features) and 7 (zero) are the gather's
+  EncodeTiledFn fn = encode_fn2();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {48, rows + 1};
+  cuuint64_t strides[1] = {96};
+  cuuint32_t box[2] = {48, 1};
+  cuuint32_t es[2] = {1, 1};
+  return fn(&f.mapX, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, f.trace16, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 bool fused_make_maps(FusedC3& f, uint64_t n) {

@@ -186,7 +186,7 @@ struct FusedC3 {
   float* T = nullptr;                 // [15][256] constant fc1 table (owned)
   __nv_bfloat16* w1p = nullptr;       // conv1 weight [64][128] in the fused row layout (owned):
                                       // per tap h: cols 0..46 attributes, 48..50 time features
-  __nv_bfloat16* trace16 = nullptr;   // per-run bf16 copy of the rank's trace rows [rows][64] (owned)
+  __nv_bfloat16* trace16 = nullptr;   // per-run bf16 copy of the rank's trace rows [rows + 1][48] (owned)
   size_t trace16_cap = 0;
   const float* head_w = nullptr;      // fc2 [3][256]
   const float* head_b = nullptr;
@@ -198,7 +198,7 @@ struct FusedC3 {
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
   CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
-  CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][64] (box 64 x 1, SWIZZLE_128B)
+  CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][48] (box 48 x 1, SWIZZLE_128B)
   uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)
 };
 void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);

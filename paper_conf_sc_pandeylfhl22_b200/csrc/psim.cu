@@ -815,7 +815,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   }
   if (fused && n) {
     // bf16 operand rows of the rank's trace (once per run; the trace crosses HBM once more)
-    const size_t t16 = (size_t)rows * 128;
+    const size_t t16 = (size_t)rows * 96;
     if (ctx->fused.trace16_cap < t16) {
       dfree(ctx->fused.trace16);
       ctx->fused.trace16 = nullptr;
@@ -823,7 +823,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       ctx->fused.trace16_cap = t16;
     }
     // row `rows` of trace16 is all zero: the padding rows of the gathered input point at it
-    CK(cudaMemsetAsync(ctx->fused.trace16 + (size_t)rows * 64, 0, 128, st));
+    CK(cudaMemsetAsync(ctx->fused.trace16 + (size_t)rows * 48, 0, 96, st));
     if (!fused_make_trace_map(ctx->fused, (uint64_t)rows))
       FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for the trace gather map");
     if (stream_load) {
