@@ -54,9 +54,7 @@ constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
 constexpr int THREADS = 416;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 gather
 constexpr int MMA_WARP = 8, GATHER_WARP0 = 9;
-#ifndef PSIM_GATHER_DEPTH
-#define PSIM_GATHER_DEPTH 1        // items issued ahead of the one being completed
-#endif
+
 }  // namespace cs
 
 struct ConvArgs {
@@ -120,7 +118,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
-  uint64_t* xfull = bars + 24;     // [NX] 4 gather warps
+  uint64_t* xfull = bars + 24;     // [NX] 4 gather warps (arrive.expect_tx) + the gathered rows (complete_tx)
   uint64_t* xempty = bars + 28;    // [NX] commit
   uint64_t* c1full = bars + 4;     // [2] commit
   uint64_t* c1empty = bars + 6;    // [2] 4 (EG-A)
@@ -135,13 +133,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
-  uint64_t* xtma = bars + 32;      // [NX] 4 gather warps (expect_tx) + the gathered rows (complete_tx)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 36);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (tid == 0) {
-    for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); mbar_init(xtma + i, 4); }
+    for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); }
     for (int i = 0; i < 2; ++i) {
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 4);
@@ -359,10 +356,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // tile::gather4 (4 arbitrary trace16 rows per instruction, SWIZZLE_128B applied
     // on the way): padding rows point at the all-zero row past the rank's rows, the
     // current instruction at its own row (time features 0), context rows at the row
-    // of their queue entry.  Once an item's rows have landed (xtma), the owner
-    // threads overwrite chunk 6 of their context rows with the time features and
-    // signal xfull.  Two items are in flight: item n is issued before item n-1 is
-    // completed.  No load result is consumed in the iteration that issues it: block
+    // of their queue entry.  The owner threads write chunk 6 (time features) and
+    // fence it, then each gather warp arrives on the slot's xfull barrier with the
+    // byte count its TMA gathers will deliver (expect_tx): xfull completes the moment
+    // the last row lands, with no gather-thread round trip.  Up to NX items are in
+    // flight, limited only by the MMA freeing slots.  No load result is consumed in the iteration that issues it: block
     // ids of tile t+2 are loaded at position 0 of tile t, their sub-trace state at
     // position 2, queue entries of item n+2 during item n.
     const int m = tid - cs::GATHER_WARP0 * 32;
@@ -416,18 +414,6 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     Ent ea, eb, ea2, eb2;                             // raw queue parts of items n, n+1
     if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
     if (n_items > 1) { stage_a(m0, 1, 0, ea2); stage_a(m0, 1, 1, eb2); }
-    // time chunks of the items issued but not completed yet (n-1, n-2)
-    uint2 pA1 = make_uint2(0u, 0u), pB1 = make_uint2(0u, 0u), pA2 = pA1, pB2 = pA1;
-    // item n-1 landed -> time features of its context rows -> visible to tcgen05 -> xfull
-    auto complete = [&](uint32_t nprev, uint2 pA, uint2 pB) {
-      const int sp = (int)(nprev % cs::NX);
-      wait_full(xtma + sp, nprev / cs::NX);
-      uint8_t* xp = sm + cs::X_OFF + sp * 32768;
-      (void)xp; (void)pA; (void)pB;
-      fence_async_smem();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(xfull + sp);
-    };
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
@@ -448,7 +434,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         // writes only chunks 0..5, so this can go in before the rows land
         st_sw128(xa, m, 6, make_uint4(tA.x, tA.y, 0u, 0u));
         st_sw128(xa + 16384, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));
-        if (lane == 0) mbar_expect_tx(xtma + xs, 64 * 96);    // this warp's 64 rows, 96 B each
+        fence_async_smem();                               // chunk 6 visible to tcgen05
+        __syncwarp();
+        if (lane == 0) mbar_expect_tx(xfull + xs, 64 * 96);   // arrive + this warp's 64 rows of 96 B
         __syncwarp();
         // lane l < 16 fetches rows (atom h = l >> 3) of blocks 32 wq + 4 g .. + 3, g = l & 7
         const int g = lane & 7, h = (lane >> 3) & 1;
@@ -460,7 +448,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           r4[t] = h ? vb : va;
         }
         if (lane < 16)
-          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xtma + xs, 0, r4[0], r4[1], r4[2], r4[3]);
+          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4[0], r4[1], r4[2], r4[3]);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
       ea = ea2; eb = eb2;                             // item n+1's raw queue entries
@@ -469,20 +457,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         stage_a(mm, (j + 2) & 3, 0, ea2); stage_a(mm, (j + 2) & 3, 1, eb2);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
-#if PSIM_GATHER_DEPTH == 2
-      if (nI > 1) complete(nI - 2, pA2, pB2);       // item n-2 landed long ago
-      pA2 = pA1; pB2 = pB1;
-#else
-      if (nI > 0) complete(nI - 1, pA1, pB1);
-#endif
-      pA1 = tA; pB1 = tB;
       if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
       if (j == 3) { m0 = m1; m1 = m2; }               // next tile
     }
-#if PSIM_GATHER_DEPTH == 2
-    if (n_items > 1) complete(n_items - 2, pA2, pB2);
-#endif
-    if (n_items > 0) complete(n_items - 1, pA1, pB1);   // the last item
   }
   fence_before();
   __syncthreads();
