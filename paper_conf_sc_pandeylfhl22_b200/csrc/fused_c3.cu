@@ -44,11 +44,15 @@ constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
 constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
 constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of W3, streamed by TMA
                                              // (halves alternate with the conv3 MMAs, from L2)
-constexpr int NX = 3;                        // X slots: gathered items in flight
+constexpr int NX = 2;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
 constexpr int A2_OFF = X_OFF + NX * 32 * 1024;   // 1 atom  [128][64]
 constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
-constexpr int BAR_OFF = A3_OFF + 32 * 1024;  // mbarriers
+// gather metadata staged by cp.async (no register waits on loads in flight):
+constexpr int SID_OFF = A3_OFF + 32 * 1024;  // u32   [4 tiles][128]    block ids
+constexpr int SMETA_OFF = SID_OFF + 2048;    // uint4 [4 tiles][128]    {id, k, ws lo, Clock lo}
+constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [4 items][128][2] queue entries of rows 2j, 2j+1
+constexpr int BAR_OFF = SENT_OFF + 16384;    // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
@@ -316,115 +320,145 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         if (lane == 0) { mbar_arrive(c2empty + h); mbar_arrive(a3full); }
         if (q == 0) PSIM_TS(59 + 4 * h);
       }
-      // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p] (256-B row per thread, straight from
-      // registers; the TMA unit stays free for the row gathers)
+      // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p].  Each warp stages its 32 rows (256 B
+      // each) in exactly the A3 bytes it writes itself in the next conv2 epilogue (rows
+      // 32 q .. 32 q + 31 of both atoms; the conv3 MMAs that read A3 have completed), so no
+      // other warp can overwrite them early; XOR-swizzled by 16-B chunk, then written out
+      // coalesced: one instruction stores two whole 256-B rows.
       const uint32_t bi = tl * cs::TILE + m;
       const uint32_t id = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
-      wait_full(c3full, it);                          // conv3 accumulated
+      wait_full(c3full, it);                          // conv3 accumulated (and A3 no longer read)
       if (q == 0) PSIM_TS(65);
       fence_after();
-      uint32_t pk[64];
-      {
-        uint32_t r0[32], r1[32];
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 32, r1);
+      // staged row r (< 32) of this warp: atom r >> 4, 256-B slot r & 15 of the warp's 4 KB there
+      auto stg = [&](int r, int c) -> uint4* {
+        return reinterpret_cast<uint4*>(sm + cs::A3_OFF + (r >> 4) * 16384 + q * 4096 + (r & 15) * 256) + (c ^ (r & 15));
+      };
+#pragma unroll 1
+      for (int half = 0; half < 2; ++half) {
+        uint32_t r0[32], r1[32], pk[32];
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64 + 32, r1);
         tmem_wait_ld();
-        bias_relu_pack32(r0, sb3, pk);
-        bias_relu_pack32(r1, sb3 + 32, pk + 16);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 96, r1);
-        tmem_wait_ld();
-        bias_relu_pack32(r0, sb3 + 64, pk + 32);
-        bias_relu_pack32(r1, sb3 + 96, pk + 48);
+        bias_relu_pack32(r0, sb3 + half * 64, pk);
+        bias_relu_pack32(r1, sb3 + half * 64 + 32, pk + 16);
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+          *stg(lane, half * 8 + c) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
       }
       fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(c3empty);            // C3 TMEM free for the next tile's conv3
-      if (id != 0xFFFFFFFFu) {
-        uint4* dst = reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(id >> 4) * 14 + (id & 15)) * 128);
-#pragma unroll
-        for (int c = 0; c < 16; ++c) dst[c] = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+#pragma unroll 4
+      for (int u = 0; u < 16; ++u) {
+        const int rr = 2 * u + (lane >> 4), cc = lane & 15;
+        const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
+        const uint4 v = *stg(rr, cc);
+        if (rid != 0xFFFFFFFFu)
+          reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128)[cc] = v;
       }
+      __syncwarp();                                   // staging reads done before the next tile's A3 writes
       if (q == 0) PSIM_TS(66);
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
     // Thread m owns block m of each tile and builds its input rows 2j and 2j+1 for
     // the 4 conv1 positions j (items).  Operand row layout (per input row, 64 bf16):
     // cols 0..46 the trace attributes, col 47 zero, cols 48..50 the time features,
-    // cols 51..63 zero.  The 128-B rows are fetched by the TMA unit with
+    // cols 51..63 zero.  The 96-B rows are fetched by the TMA unit with
     // tile::gather4 (4 arbitrary trace16 rows per instruction, SWIZZLE_128B applied
     // on the way): padding rows point at the all-zero row past the rank's rows, the
     // current instruction at its own row (time features 0), context rows at the row
     // of their queue entry.  The owner threads write chunk 6 (time features) and
     // fence it, then each gather warp arrives on the slot's xfull barrier with the
-    // byte count its TMA gathers will deliver (expect_tx): xfull completes the moment
-    // the last row lands, with no gather-thread round trip.  Up to NX items are in
-    // flight, limited only by the MMA freeing slots.  No load result is consumed in the iteration that issues it: block
-    // ids of tile t+2 are loaded at position 0 of tile t, their sub-trace state at
-    // position 2, queue entries of item n+2 during item n.
+    // byte count its TMA gathers will deliver (expect_tx).
+    //
+    // The metadata chain block id -> sub-trace state -> queue entries is staged in
+    // shared memory by cp.async, one stage per tile or item ahead, so no register
+    // ever waits on a load in flight: iteration n (tile t, item j) issues the block
+    // ids of tile t+3 and the states of tile t+2 (j == 0) and the queue entries of
+    // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1:
+    // one group per iteration).
     const int m = tid - cs::GATHER_WARP0 * 32;
     const int wq = warp - cs::GATHER_WARP0;          // gather warp 0..3: tile rows 32 wq .. 32 wq + 31
-    // Every load below is UNCONDITIONAL (out-of-range lanes read a clamped, valid
-    // address) and lands in a register of its own: a predicated load merged into a
-    // pre-set value would make the merge wait for the load where it is issued.
-    struct Meta { uint32_t id; int k; uint32_t i, clo; bool valid; };
-    struct Ent { uint4 v; int kind; };               // kind: 0 padding, 1 current, 2 context
-    auto meta_ids = [&](uint32_t tl, Meta& mt) {         // stage 1: block id
-      const uint32_t bi = tl * cs::TILE + m;
-      mt.valid = tl < ntiles && bi < nblocks;
-      mt.id = a.blocks[mt.valid ? bi : 0u];              // nblocks > 0 whenever this runs
+    uint32_t* sIds = reinterpret_cast<uint32_t*>(sm + cs::SID_OFF);
+    uint4* sMeta = reinterpret_cast<uint4*>(sm + cs::SMETA_OFF);
+    uint4* sEnt = reinterpret_cast<uint4*>(sm + cs::SENT_OFF);
+    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const uint32_t n_items = my_tiles * 4;
+    auto valid_of = [&](uint32_t T) -> bool {         // block m of this CTA's T-th tile exists
+      const uint32_t tl = blockIdx.x + T * gridDim.x;
+      return T < my_tiles && tl * cs::TILE + m < nblocks;
     };
-    auto meta_state = [&](Meta& mt) {                    // stage 2: sub-trace state
-      const uint32_t b = mt.id >> 4;
-      mt.k = a.count[b];
-      mt.i = (uint32_t)a.ws[b];                          // + step at use
-      mt.clo = (uint32_t)a.clock[b];
+    auto stage_ids = [&](uint32_t T) {                // stage 1: block id of tile T
+      if (valid_of(T)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
     };
-    auto stage_a = [&](const Meta& mt, int j, int h, Ent& en) {   // raw queue entry of row 2j+h
-      const int R = (int)(mt.id & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
-      en.kind = (mt.valid && R <= mt.k) ? (R == 0 ? 1 : 2) : 0;
-      const int ent = en.kind == 2 ? mt.k - R : 0;        // context newest first (R6)
-      en.v = a.q[(uint64_t)ent * a.qn + (mt.id >> 4)];
+    auto stage_meta = [&](uint32_t T) {               // stage 2: sub-trace state of tile T (ids landed)
+      if (!valid_of(T)) return;
+      const uint32_t id = sIds[(T & 3) * 128 + m];
+      const uint32_t b = id >> 4;
+      uint4* d = sMeta + (T & 3) * 128 + m;
+      reinterpret_cast<uint32_t*>(d)[0] = id;
+      cp_async4(reinterpret_cast<uint32_t*>(d) + 1, a.count + b);
+      cp_async4(reinterpret_cast<uint32_t*>(d) + 2, a.ws + b);        // low word (little endian)
+      cp_async4(reinterpret_cast<uint32_t*>(d) + 3, a.clock + b);
+    };
+    auto stage_ent = [&](uint32_t n) {                // stage 3: queue entries of item n (states landed)
+      const uint32_t T = n >> 2;
+      if (!valid_of(T)) return;
+      const int j = (int)(n & 3);
+      const uint4 mt = sMeta[(T & 3) * 128 + m];
+      const int k = (int)mt.y;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int R = (int)(mt.x & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
+        if (R >= 1 && R <= k)                              // context row: entry k - R (newest first, R6)
+          cp_async16(sEnt + ((n & 3) * 128 + m) * 2 + h, a.q + (uint64_t)(k - R) * a.qn + (mt.x >> 4));
+      }
     };
     // One input row: the trace16 row the TMA fetches, and the time-feature chunk
-    // (cols 48..55) written after it lands (context rows only, R2).
-    auto row_of = [&](const Ent& en, const Meta& mt, uint2& tchunk) -> uint32_t {
+    // (cols 48..55) written next to it (context rows only, R2).
+    auto row_of = [&](bool valid, const uint4& mt, int R, const uint4& ev, uint2& tchunk) -> uint32_t {
       tchunk = make_uint2(0u, 0u);
-      if (en.kind == 0) return a.zero_row;             // zero padding at the tail
-      if (en.kind == 1) return (uint32_t)((int64_t)(mt.i + (uint32_t)a.step) - a.row_lo);   // current first
-      const int c = en.v.z & 0xFFFF, sv = (en.v.z >> 16) & 0xFFFF;
-      const int age = (int)(mt.clo - en.v.y);
+      const int k = (int)mt.y;
+      if (!valid || R > k) return a.zero_row;                 // zero padding at the tail
+      if (R == 0) return (uint32_t)((int64_t)(mt.z + (uint32_t)a.step) - a.row_lo);   // current first
+      const int c = ev.z & 0xFFFF, sv = (ev.z >> 16) & 0xFFFF;
+      const int age = (int)(mt.w - ev.y);
       const int t0 = min(age, kTimeMax), t1 = min(max(0, c - age), kTimeMax), t2 = min(c + sv - age, kTimeMax);
       tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
-      return (uint32_t)((int64_t)en.v.x - a.row_lo);
+      return (uint32_t)((int64_t)ev.x - a.row_lo);
     };
     // chunk 7 (cols 56..63) of every X row is never written by the TMA: zero it once
 #pragma unroll
     for (int s2 = 0; s2 < cs::NX; ++s2)
 #pragma unroll
       for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
-    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    const uint32_t n_items = my_tiles * 4;
-    Meta m0, m1, m2;                                  // tiles it, it+1, it+2
-    meta_ids(blockIdx.x, m0);
-    meta_ids(blockIdx.x + gridDim.x, m1);
-    meta_state(m0);
-    meta_state(m1);
-    Ent ea, eb, ea2, eb2;                             // raw queue parts of items n, n+1
-    if (n_items > 0) { stage_a(m0, 0, 0, ea); stage_a(m0, 0, 1, eb); }
-    if (n_items > 1) { stage_a(m0, 1, 0, ea2); stage_a(m0, 1, 1, eb2); }
+    // prologue: ids of tiles 0..2, states of tiles 0..1, entries of items 0..1
+    for (uint32_t T = 0; T < 3; ++T) stage_ids(T);
+    cp_async_commit();
+    cp_async_wait<0>();
+    for (uint32_t T = 0; T < 2; ++T) stage_meta(T);
+    cp_async_commit();
+    cp_async_wait<0>();
+    stage_ent(0);
+    stage_ent(1);
+    cp_async_commit();
+    cp_async_commit();   // two groups so that wait_group 1 at item 0 covers the entries of item 0
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
-      const int j = (int)(nI & 3), s = j & 1;
-      if (j == 0) meta_ids(blockIdx.x + (it + 2) * gridDim.x, m2);
-      if (j == 2) meta_state(m2);
+      const int j = (int)(nI & 3);
+      cp_async_wait<1>();                             // everything staged up to iteration nI - 2 has landed
       if (j == 0 && warp == cs::GATHER_WARP0) PSIM_TS(80);
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      const bool valid = valid_of(it);
+      const uint4 mt = sMeta[(it & 3) * 128 + m];
+      const uint4 e0 = sEnt[((nI & 3) * 128 + m) * 2], e1 = sEnt[((nI & 3) * 128 + m) * 2 + 1];
+      const int R0 = (int)(mt.x & 15) * 8 + 2 * j;
       uint2 tA, tB;
-      const uint32_t rA = row_of(ea, m0, tA);
-      const uint32_t rB = row_of(eb, m0, tB);
+      const uint32_t rA = row_of(valid, mt, R0, e0, tA);
+      const uint32_t rB = row_of(valid, mt, R0 + 1, e1, tB);
       const int xs = (int)(nI % cs::NX);
       wait_empty(xempty + xs, nI / cs::NX);
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
@@ -451,15 +485,13 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4[0], r4[1], r4[2], r4[3]);
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
-      ea = ea2; eb = eb2;                             // item n+1's raw queue entries
-      if (nI + 2 < n_items) {                         // raw queue entries of item n+2
-        const Meta& mm = j >= 2 ? m1 : m0;
-        stage_a(mm, (j + 2) & 3, 0, ea2); stage_a(mm, (j + 2) & 3, 1, eb2);
-      }
+      // stage the metadata of later iterations
+      if (j == 0) { stage_ids(it + 3); stage_meta(it + 2); }
+      if (nI + 2 < n_items) stage_ent(nI + 2);
+      cp_async_commit();
       if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
-      if (j == 3) { m0 = m1; m1 = m2; }               // next tile
     }
+    cp_async_wait<0>();
   }
   fence_before();
   __syncthreads();
