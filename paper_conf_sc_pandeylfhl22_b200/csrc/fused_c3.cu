@@ -20,13 +20,15 @@
 //
 // conv_stack_kernel roles (448 threads): warps 0..3 = EG-A (conv1 epilogue:
 // TMEM -> bias, ReLU, bf16 -> A2), warps 4..7 = EG-B (conv2 epilogue -> A3,
-// conv3 epilogue -> staging rows), warp 8 = TMEM allocator, lane 0 the
-// single-thread tcgen05.mma issuer, lane 1 the W3 streamer; warps 9..12 =
-// gather (cp.async of bf16 trace rows + time features straight into the
-// SWIZZLE_128B X tile); warp 13 = a4 write-back (TMA bulk stores, one per
-// sub-trace run).  W1/W2 stay resident in smem (48 KB); W3 (64 KB) is streamed
-// one K-half (32 KB) at a time from L2, alternating with the conv3 MMAs, which
-// frees a dedicated 32 KB staging buffer.  Per 128-block tile the MMA order is
+// conv3 epilogue -> a4 rows, staged in its own A3 bytes and stored coalesced),
+// warp 8 = TMEM allocator, lane 0 the single-thread tcgen05.mma issuer;
+// warps 9..12 = gather (metadata staged in smem by cp.async, trace rows by TMA
+// tile::gather4 straight into the SWIZZLE_128B X tile, time features by the
+// owner threads); warp 13 lane 0 = W3 streamer (its own warp: a spinning
+// mbarrier wait must never share a warp with the MMA issuer).  W1/W2 stay
+// resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at a
+// time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
+// order is
 //   c1(0) c1(1) [c3(prev,1)] c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1)
 // with K-split accumulation so A2 (16 KB) and A3 (32 KB) are single buffers.
 #include "internal.h"
@@ -46,18 +48,21 @@ constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of
                                              // (halves alternate with the conv3 MMAs, from L2)
 constexpr int NX = 2;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
-constexpr int A2_OFF = X_OFF + NX * 32 * 1024;   // 1 atom  [128][64]
-constexpr int A3_OFF = A2_OFF + 16 * 1024;   // 2 atoms [128][64]
+constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][256 B]
 // gather metadata staged by cp.async (no register waits on loads in flight):
-constexpr int SID_OFF = A3_OFF + 32 * 1024;  // u32   [4 tiles][128]    block ids
+constexpr int SID_OFF = STG_OFF + 32 * 1024; // u32   [4 tiles][128]    block ids
 constexpr int SMETA_OFF = SID_OFF + 2048;    // uint4 [4 tiles][128]    {id, k, ws lo, Clock lo}
 constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [4 items][128][2] queue entries of rows 2j, 2j+1
 constexpr int BAR_OFF = SENT_OFF + 16384;    // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
-constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;   // C1 x2, C2 x2, C3
-constexpr int THREADS = 416;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 gather
-constexpr int MMA_WARP = 8, GATHER_WARP0 = 9;
+// C1 x2 (64 fp32 each), C2 x2 (128 fp32 each), C3 (128 fp32).  The conv2 / conv3 A operands
+// (bf16 activations of conv1 / conv2) are written back by the epilogues into the first
+// 32 / 64 columns of the slot they were read from (packed bf16x2) and read by the MMA
+// from TMEM: no smem traffic for A2 / A3.
+constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;
+constexpr int THREADS = 448;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 gather, 13 W3
+constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, W3_WARP = 13;
 
 }  // namespace cs
 
@@ -124,14 +129,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
   uint64_t* xfull = bars + 24;     // [NX] 4 gather warps (arrive.expect_tx) + the gathered rows (complete_tx)
   uint64_t* xempty = bars + 28;    // [NX] commit
-  uint64_t* c1full = bars + 4;     // [2] commit
-  uint64_t* c1empty = bars + 6;    // [2] 4 (EG-A)
-  uint64_t* a2full = bars + 8;     //     4 (EG-A)
-  uint64_t* a2empty = bars + 9;    //     commit
+  uint64_t* c1full = bars + 4;     // [2] commit: conv1 of the slot's item done
+  uint64_t* c1empty = bars + 6;    // [2] commit: the conv2 MMAs reading the slot's A2 done
+  uint64_t* a2full = bars + 8;     // [2] 4 (EG-A): A2 (bf16) written into the C1 slot
   uint64_t* c2full = bars + 10;    // [2] commit (one TMEM slot per conv2 position)
-  uint64_t* c2empty = bars + 12;   // [2] 4 (EG-B)
-  uint64_t* a3full = bars + 14;    //     4 (EG-B)
-  uint64_t* a3empty = bars + 15;   //     commit
+  uint64_t* c2empty = bars + 12;   // [2] commit: the conv3 MMAs reading the slot's A3 done
+  uint64_t* a3full = bars + 14;    // [2] 4 (EG-B): A3 (bf16) written into the C2 slot
   uint64_t* c3full = bars + 16;    //     commit
   uint64_t* c3empty = bars + 17;   //     4 (EG-B)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
@@ -144,11 +147,10 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   if (tid == 0) {
     for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); }
     for (int i = 0; i < 2; ++i) {
-      mbar_init(c1full + i, 1); mbar_init(c1empty + i, 4);
-      mbar_init(c2full + i, 1); mbar_init(c2empty + i, 4);
+      mbar_init(c1full + i, 1); mbar_init(c1empty + i, 1); mbar_init(a2full + i, 4);
+      mbar_init(c2full + i, 1); mbar_init(c2empty + i, 1); mbar_init(a3full + i, 4);
     }
-    mbar_init(a2full, 4); mbar_init(a2empty, 1);
-    mbar_init(a3full, 4); mbar_init(a3empty, 1); mbar_init(c3full, 1); mbar_init(c3empty, 4);
+    mbar_init(c3full, 1); mbar_init(c3empty, 4);
     mbar_init(wbar, 1);
     mbar_init(w3full, 1); mbar_init(w3empty, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -201,32 +203,32 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         mma_commit(xempty + xs);
         mma_commit(c1full + s);
       };
-      auto c2 = [&](uint32_t it, int h, int kh) {
+      auto c2 = [&](uint32_t it, int h, int kh) {   // conv2 position h, K-half kh = item 2h+kh (C1 slot kh)
         PSIM_TS(8 + 2 * (h * 2 + kh));
-        wait_full(a2full, it * 4 + h * 2 + kh);
+        wait_full(a2full + kh, it * 2 + h);
         if (kh == 0) wait_empty(c2empty + h, it);
         PSIM_TS(9 + 2 * (h * 2 + kh));
         fence_after();
 #pragma unroll
         for (int k = 0; k < 4; ++k)
-          mma_bf16(tmem + cs::TMEM_C2 + h * 128, sw128_desc(sbase + cs::A2_OFF + k * 32),
-                   sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
-        mma_commit(a2empty);
+          mma_bf16_ts(tmem + cs::TMEM_C2 + h * 128, tmem + cs::TMEM_C1 + kh * 64 + 8 * k,
+                      sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
+        mma_commit(c1empty + kh);   // C1 slot kh (its A2) free for conv1 two items later
         if (kh == 1) mma_commit(c2full + h);
       };
-      auto c3 = [&](uint32_t it, int kh) {   // the (2 it + kh)-th conv3 MMA group uses W3 K-half kh
+      auto c3 = [&](uint32_t it, int kh) {   // the (2 it + kh)-th conv3 MMA group: W3 K-half kh, A3 in C2 slot kh
         PSIM_TS(16 + 2 * kh);
-        wait_full(a3full, it * 2 + kh);
+        wait_full(a3full + kh, it);
         if (kh == 0) wait_empty(c3empty, it);
         wait_full(w3full, it * 2 + kh);
         PSIM_TS(17 + 2 * kh);
         fence_after();
 #pragma unroll
         for (int k = 0; k < 8; ++k)
-          mma_bf16(tmem + cs::TMEM_C3, sw128_desc(sbase + cs::A3_OFF + (k >> 2) * 16384 + (k & 3) * 32),
-                   sw128_desc(sbase + cs::W3_OFF + (k >> 2) * 16384 + (k & 3) * 32), id128, (kh | k) != 0);
-        mma_commit(a3empty);
+          mma_bf16_ts(tmem + cs::TMEM_C3, tmem + cs::TMEM_C2 + kh * 128 + 8 * k,
+                      sw128_desc(sbase + cs::W3_OFF + (k >> 2) * 16384 + (k & 3) * 32), id128, (kh | k) != 0);
         mma_commit(w3empty);
+        mma_commit(c2empty + kh);   // C2 slot kh free for the next tile's conv2 position kh
         if (kh == 1) mma_commit(c3full);
       };
       uint32_t it = 0;
@@ -236,20 +238,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         c2(it, 0, 0); c2(it, 0, 1); c1(it, 2); c1(it, 3); c3(it, 0); c2(it, 1, 0); c2(it, 1, 1);
       }
       if (it > 0) c3(it - 1, 1);
-    } else if (lane == 1) {   // ============================ W3 streamer
-      // conv3 MMA groups alternate K-halves 0, 1, 0, 1, ...; fill n waits until the
-      // MMAs of fill n-1 have finished reading the buffer, then loads half n & 1
-      uint32_t nfill = 0;
-      for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) nfill += 2;
-      for (uint32_t f = 0; f < nfill; ++f) {
-        wait_empty(w3empty, f);
-        mbar_expect_tx(w3full, 32 * 1024);
-        for (int a2 = 0; a2 < 2; ++a2)
-          tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (f & 1) + a2) * 64, 0);
-      }
     }
     __syncwarp();
-  } else if (warp < 4) {   // ============================ EG-A: conv1 epilogues (C1 -> A2)
+  } else if (warp < 4) {   // ============================ EG-A: conv1 epilogues (C1 -> A2, in TMEM)
     const int q = warp & 3;
     const int m = q * 32 + lane;                    // tile row = TMEM lane
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
@@ -271,18 +262,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           bias_relu_pack32(r0, sb1, pk);
           bias_relu_pack32(r1, sb1 + 32, pk + 16);
         }
+        if (q == 0) PSIM_TS(34 + 4 * j);
+        // A2 = relu(C1 + b1) as bf16x2 into columns 0..31 of the same C1 slot (conv2's A operand)
+        tmem_st16(tmem + lane_base + cs::TMEM_C1 + s * 64, pk);
+        tmem_st16(tmem + lane_base + cs::TMEM_C1 + s * 64 + 16, pk + 16);
+        tmem_wait_st();
         fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(c1empty + s);
-        if (q == 0) PSIM_TS(34 + 4 * j);
-        wait_empty(a2empty, it * 4 + j);
-        if (q == 0) PSIM_TS(35 + 4 * j);
-#pragma unroll
-        for (int c = 0; c < 8; ++c)
-          st_sw128(sm + cs::A2_OFF, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
-        fence_async_smem();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(a2full);
+        if (lane == 0) mbar_arrive(a2full + s);
         if (q == 0) PSIM_TS(48 + j);
       }
     }
@@ -293,47 +280,41 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     uint32_t it = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
 #pragma unroll 1
-      for (int h = 0; h < 2; ++h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (2 atoms)
+      for (int h = 0; h < 2; ++h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (same slot)
         if (q == 0) PSIM_TS(56 + 4 * h);
         wait_full(c2full + h, it);
         if (q == 0) PSIM_TS(57 + 4 * h);
         fence_after();
-        wait_empty(a3empty, it * 2 + h);
-        if (q == 0) PSIM_TS(58 + 4 * h);
 #pragma unroll 1
-        for (int cp = 0; cp < 2; ++cp) {
+        for (int cp = 0; cp < 2; ++cp) {   // channels 64 cp .. 64 cp + 63 -> A3 columns 32 cp .. 32 cp + 31
           uint32_t r0[32], r1[32];
           tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
           tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
           tmem_wait_ld();
-          uint8_t* atom = sm + cs::A3_OFF + cp * 16384;   // 64 channels per atom
           uint32_t pk[32];
           bias_relu_pack32(r0, sb2 + cp * 64, pk);
           bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
-#pragma unroll
-          for (int c = 0; c < 8; ++c)
-            st_sw128(atom, m, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
+          // in place: columns 32 cp .. 32 cp + 31 were read already (cp = 1 reads 64 .. 127)
+          tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32, pk);
+          tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32 + 16, pk + 16);
         }
+        tmem_wait_st();
         fence_before();
-        fence_async_smem();
         __syncwarp();
-        if (lane == 0) { mbar_arrive(c2empty + h); mbar_arrive(a3full); }
+        if (lane == 0) mbar_arrive(a3full + h);
         if (q == 0) PSIM_TS(59 + 4 * h);
       }
       // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p].  Each warp stages its 32 rows (256 B
-      // each) in exactly the A3 bytes it writes itself in the next conv2 epilogue (rows
-      // 32 q .. 32 q + 31 of both atoms; the conv3 MMAs that read A3 have completed), so no
-      // other warp can overwrite them early; XOR-swizzled by 16-B chunk, then written out
-      // coalesced: one instruction stores two whole 256-B rows.
+      // each) in its own 8 KB of the staging buffer, XOR-swizzled by 16-B chunk, then writes
+      // them out coalesced: one instruction stores two whole 256-B rows.
       const uint32_t bi = tl * cs::TILE + m;
       const uint32_t id = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
-      wait_full(c3full, it);                          // conv3 accumulated (and A3 no longer read)
+      wait_full(c3full, it);                          // conv3 accumulated
       if (q == 0) PSIM_TS(65);
       fence_after();
-      // staged row r (< 32) of this warp: atom r >> 4, 256-B slot r & 15 of the warp's 4 KB there
-      auto stg = [&](int r, int c) -> uint4* {
-        return reinterpret_cast<uint4*>(sm + cs::A3_OFF + (r >> 4) * 16384 + q * 4096 + (r & 15) * 256) + (c ^ (r & 15));
+      auto stg = [&](int r, int c) -> uint4* {   // staged row r (< 32) of this warp, 16-B chunk c
+        return reinterpret_cast<uint4*>(sm + cs::STG_OFF + q * 8192 + r * 256) + (c ^ (r & 15));
       };
 #pragma unroll 1
       for (int half = 0; half < 2; ++half) {
@@ -341,12 +322,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64, r0);
         tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64 + 32, r1);
         tmem_wait_ld();
+        if (q == 0) PSIM_TS(68 + half);
         bias_relu_pack32(r0, sb3 + half * 64, pk);
         bias_relu_pack32(r1, sb3 + half * 64 + 32, pk + 16);
 #pragma unroll
         for (int c = 0; c < 8; ++c)
           *stg(lane, half * 8 + c) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
       }
+      if (q == 0) PSIM_TS(67);
       fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(c3empty);            // C3 TMEM free for the next tile's conv3
@@ -360,6 +343,19 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       }
       __syncwarp();                                   // staging reads done before the next tile's A3 writes
       if (q == 0) PSIM_TS(66);
+    }
+  } else if (warp == cs::W3_WARP) {
+    if (lane == 0) {   // ============================ W3 streamer
+      // conv3 MMA groups alternate K-halves 0, 1, 0, 1, ...; fill n waits until the
+      // MMAs of fill n-1 have finished reading the buffer, then loads half n & 1
+      uint32_t nfill = 0;
+      for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) nfill += 2;
+      for (uint32_t f = 0; f < nfill; ++f) {
+        wait_empty(w3empty, f);
+        mbar_expect_tx(w3full, 32 * 1024);
+        for (int a2 = 0; a2 < 2; ++a2)
+          tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (f & 1) + a2) * 64, 0);
+      }
     }
   } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
     // Thread m owns block m of each tile and builds its input rows 2j and 2j+1 for

@@ -18,7 +18,7 @@ for j in range(4):
 for h in range(2):
     names[56 + 4 * h] = f"e2({h})wait"; names[57 + 4 * h] = f"e2({h})C2"; names[58 + 4 * h] = f"e2({h})A3free"
     names[59 + 4 * h] = f"e2({h})done"
-names.update({64: "e3wait", 65: "e3C3", 66: "e3done", 80: "g start"})
+names.update({64: "e3wait", 65: "e3C3", 66: "e3done", 67: "e3staged", 68: "e3ld0", 69: "e3ld1", 80: "g start"})
 for j in range(4):
     names[81 + 3 * j] = f"g{j}a"; names[82 + 3 * j] = f"g{j}slot"; names[83 + 3 * j] = f"g{j}xfull(prev)"
 for j in range(4):
