@@ -18,19 +18,20 @@
 // folded into T[P] = b_fc1 + sum_{p >= P} Wfc1[:, p] c3 (R18).
 // P_b = ceil((k_b + 1) / 8).  Exact in real arithmetic; the oracle stays dense.
 //
-// conv_stack_kernel roles (448 threads): warps 0..3 = EG-A (conv1 epilogue:
+// conv_stack_kernel roles (512 threads): warps 0..3 = EG-A (conv1 epilogue:
 // TMEM -> bias, ReLU, bf16 -> A2), warps 4..7 = EG-B (conv2 epilogue -> A3,
-// conv3 epilogue -> a4 rows, staged in its own A3 bytes and stored coalesced),
+// conv3 epilogue -> a4 rows, staged in smem and stored coalesced),
 // warp 8 = TMEM allocator, lane 0 the single-thread tcgen05.mma issuer;
-// warps 9..12 = gather (metadata staged in smem by cp.async, trace rows by TMA
-// tile::gather4 straight into the SWIZZLE_128B X tile, time features by the
-// owner threads); warp 13 lane 0 = W3 streamer (its own warp: a spinning
-// mbarrier wait must never share a warp with the MMA issuer).  W1/W2 stay
+// warps 9..12 = TMA row issuers (trace rows by tile::gather4 straight into the
+// SWIZZLE_128B X tile, time features from the row ring written by the
+// builders); warp 13 lane 0 = W3 streamer (its own warp: a spinning mbarrier
+// wait must never share a warp with the MMA issuer); warps 14..15 = row
+// builders (block id -> state -> queue entries -> row indices + time features).  W1/W2 stay
 // resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at a
 // time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
 // order is
 //   c1(0) c1(1) [c3(prev,1)] c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1)
-// with K-split accumulation so A2 (16 KB) and A3 (32 KB) are single buffers.
+// with K-split accumulation; the conv2 / conv3 A operands live in TMEM.
 #include "internal.h"
 #include "sim_common.cuh"
 #include "tc_common.cuh"
@@ -46,23 +47,29 @@ constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
 constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
 constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of W3, streamed by TMA
                                              // (halves alternate with the conv3 MMAs, from L2)
-constexpr int NX = 2;                        // X slots: gathered items in flight
+constexpr int NX = 3;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
-constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][256 B]
+constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][128 B] (half rows)
 // gather metadata staged by cp.async (no register waits on loads in flight):
-constexpr int SID_OFF = STG_OFF + 32 * 1024; // u32   [4 tiles][128]    block ids
+constexpr int SID_OFF = STG_OFF + 16 * 1024; // u32   [4 tiles][128]    block ids
 constexpr int SMETA_OFF = SID_OFF + 2048;    // uint4 [4 tiles][128]    {id, k, ws lo, Clock lo}
-constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [4 items][128][2] queue entries of rows 2j, 2j+1
-constexpr int BAR_OFF = SENT_OFF + 16384;    // mbarriers
+constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [3 items][128][2] queue entries of rows 2j, 2j+1 (item n in slot n % 3)
+constexpr int RQ = 3;                        // row ring: items built ahead of the TMA issue
+constexpr int RROW_OFF = SENT_OFF + 3 * 4096; // u32   [RQ][2][128] trace16 row of input row 2j+h of block m
+constexpr int RT_OFF = RROW_OFF + RQ * 1024; // uint2 [RQ][2][128] its time-feature chunk
+constexpr int BAR_OFF = RT_OFF + RQ * 2048;  // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
+static_assert(SMEM <= 232448, "conv_stack smem over the 227 KB opt-in limit");
 // C1 x2 (64 fp32 each), C2 x2 (128 fp32 each), C3 (128 fp32).  The conv2 / conv3 A operands
 // (bf16 activations of conv1 / conv2) are written back by the epilogues into the first
 // 32 / 64 columns of the slot they were read from (packed bf16x2) and read by the MMA
 // from TMEM: no smem traffic for A2 / A3.
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;
-constexpr int THREADS = 448;   // warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 gather, 13 W3
-constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, W3_WARP = 13;
+// warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 TMA row
+// issuers, 13 W3 streamer, 14-15 row builders (metadata -> row indices + time features)
+constexpr int THREADS = 512;
+constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, W3_WARP = 13, BUILD_WARP0 = 14;
 
 }  // namespace cs
 
@@ -140,12 +147,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 36);
+  uint64_t* rfull = bars + 32;     // [RQ] 2 builder warps: rows of the item in the ring
+  uint64_t* rempty = bars + 36;    // [RQ] 4 issuer warps: ring slot consumed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 44);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (tid == 0) {
     for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); }
+    for (int i = 0; i < cs::RQ; ++i) { mbar_init(rfull + i, 2); mbar_init(rempty + i, 4); }
     for (int i = 0; i < 2; ++i) {
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 1); mbar_init(a2full + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 1); mbar_init(a3full + i, 4);
@@ -274,76 +284,95 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       }
     }
   } else if (warp < 8) {   // ============================ EG-B: conv2 / conv3 epilogues
+    // Order per tile t: e2(t, 0), e3(t - 1), e2(t, 1).  e3(t - 1) becomes ready together
+    // with e2(t, 0) (conv3 K-half 1 of tile t-1 is issued just before conv2 of tile t);
+    // doing e2(t, 0) first lets conv3(t, 0) start while e3(t - 1) writes its rows out.
     const int q = warp & 3;
     const int m = q * 32 + lane;
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
-    uint32_t it = 0;
-    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+    auto e2 = [&](uint32_t it, int h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (same slot)
+      if (q == 0) PSIM_TS(56 + 4 * h);
+      wait_full(c2full + h, it);
+      if (q == 0) PSIM_TS(57 + 4 * h);
+      fence_after();
 #pragma unroll 1
-      for (int h = 0; h < 2; ++h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (same slot)
-        if (q == 0) PSIM_TS(56 + 4 * h);
-        wait_full(c2full + h, it);
-        if (q == 0) PSIM_TS(57 + 4 * h);
-        fence_after();
-#pragma unroll 1
-        for (int cp = 0; cp < 2; ++cp) {   // channels 64 cp .. 64 cp + 63 -> A3 columns 32 cp .. 32 cp + 31
-          uint32_t r0[32], r1[32];
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
-          tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
-          tmem_wait_ld();
-          uint32_t pk[32];
-          bias_relu_pack32(r0, sb2 + cp * 64, pk);
-          bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
-          // in place: columns 32 cp .. 32 cp + 31 were read already (cp = 1 reads 64 .. 127)
-          tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32, pk);
-          tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32 + 16, pk + 16);
-        }
-        tmem_wait_st();
-        fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(a3full + h);
-        if (q == 0) PSIM_TS(59 + 4 * h);
+      for (int cp = 0; cp < 2; ++cp) {   // channels 64 cp .. 64 cp + 63 -> A3 columns 32 cp .. 32 cp + 31
+        uint32_t r0[32], r1[32];
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
+        tmem_wait_ld();
+        uint32_t pk[32];
+        bias_relu_pack32(r0, sb2 + cp * 64, pk);
+        bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
+        // in place: columns 32 cp .. 32 cp + 31 were read already (cp = 1 reads 64 .. 127)
+        tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32, pk);
+        tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32 + 16, pk + 16);
       }
-      // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p].  Each warp stages its 32 rows (256 B
-      // each) in its own 8 KB of the staging buffer, XOR-swizzled by 16-B chunk, then writes
-      // them out coalesced: one instruction stores two whole 256-B rows.
+      tmem_wait_st();
+      fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(a3full + h);
+      if (q == 0) PSIM_TS(59 + 4 * h);
+    };
+    // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p]: both halves are read out of TMEM first
+    // (C3 released at once for the next tile's conv3), then one half row (64 channels,
+    // 128 B) at a time is staged in this warp's 4 KB of the staging buffer (XOR-swizzled
+    // by 16-B chunk) and written out coalesced: one instruction stores four 128-B half rows.
+    auto e3 = [&](uint32_t it, uint32_t tl) {
       const uint32_t bi = tl * cs::TILE + m;
       const uint32_t id = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
       wait_full(c3full, it);                          // conv3 accumulated
       if (q == 0) PSIM_TS(65);
       fence_after();
-      auto stg = [&](int r, int c) -> uint4* {   // staged row r (< 32) of this warp, 16-B chunk c
-        return reinterpret_cast<uint4*>(sm + cs::STG_OFF + q * 8192 + r * 256) + (c ^ (r & 15));
-      };
-#pragma unroll 1
-      for (int half = 0; half < 2; ++half) {
-        uint32_t r0[32], r1[32], pk[32];
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + half * 64 + 32, r1);
+      uint32_t pk[64];
+      {
+        uint32_t r0[32], r1[32];
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 32, r1);
         tmem_wait_ld();
-        if (q == 0) PSIM_TS(68 + half);
-        bias_relu_pack32(r0, sb3 + half * 64, pk);
-        bias_relu_pack32(r1, sb3 + half * 64 + 32, pk + 16);
+        bias_relu_pack32(r0, sb3, pk);
+        bias_relu_pack32(r1, sb3 + 32, pk + 16);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 64, r0);
+        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 96, r1);
+        tmem_wait_ld();
+        fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(c3empty);          // C3 TMEM free for the next tile's conv3
+        bias_relu_pack32(r0, sb3 + 64, pk + 32);
+        bias_relu_pack32(r1, sb3 + 96, pk + 48);
+      }
+      if (q == 0) PSIM_TS(68);
+      auto stg = [&](int r, int c) -> uint4* {   // staged half row r (< 32) of this warp, 16-B chunk c (< 8)
+        return reinterpret_cast<uint4*>(sm + cs::STG_OFF + q * 4096 + r * 128) + (c ^ (r & 7));
+      };
+#pragma unroll
+      for (int half = 0; half < 2; ++half) {
 #pragma unroll
         for (int c = 0; c < 8; ++c)
-          *stg(lane, half * 8 + c) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
-      }
-      if (q == 0) PSIM_TS(67);
-      fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(c3empty);            // C3 TMEM free for the next tile's conv3
+          *stg(lane, c) = make_uint4(pk[32 * half + 4 * c], pk[32 * half + 4 * c + 1], pk[32 * half + 4 * c + 2],
+                                     pk[32 * half + 4 * c + 3]);
+        __syncwarp();
 #pragma unroll 4
-      for (int u = 0; u < 16; ++u) {
-        const int rr = 2 * u + (lane >> 4), cc = lane & 15;
-        const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
-        const uint4 v = *stg(rr, cc);
-        if (rid != 0xFFFFFFFFu)
-          reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128)[cc] = v;
+        for (int u = 0; u < 8; ++u) {
+          const int rr = 4 * u + (lane >> 3), cc = lane & 7;
+          const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
+          const uint4 v = *stg(rr, cc);
+          if (rid != 0xFFFFFFFFu)
+            reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128 + half * 64)[cc] = v;
+        }
+        __syncwarp();                                 // staging reads done before it is rewritten
       }
-      __syncwarp();                                   // staging reads done before the next tile's A3 writes
       if (q == 0) PSIM_TS(66);
+    };
+    uint32_t it = 0, prev_tl = 0;
+    for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+      e2(it, 0);
+      if (it > 0) e3(it - 1, prev_tl);
+      e2(it, 1);
+      prev_tl = tl;
     }
+    if (it > 0) e3(it - 1, prev_tl);
   } else if (warp == cs::W3_WARP) {
     if (lane == 0) {   // ============================ W3 streamer
       // conv3 MMA groups alternate K-halves 0, 1, 0, 1, ...; fill n waits until the
@@ -357,17 +386,13 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (f & 1) + a2) * 64, 0);
       }
     }
-  } else if (warp >= cs::GATHER_WARP0) {   // ============================ gather
-    // Thread m owns block m of each tile and builds its input rows 2j and 2j+1 for
-    // the 4 conv1 positions j (items).  Operand row layout (per input row, 64 bf16):
-    // cols 0..46 the trace attributes, col 47 zero, cols 48..50 the time features,
-    // cols 51..63 zero.  The 96-B rows are fetched by the TMA unit with
-    // tile::gather4 (4 arbitrary trace16 rows per instruction, SWIZZLE_128B applied
-    // on the way): padding rows point at the all-zero row past the rank's rows, the
-    // current instruction at its own row (time features 0), context rows at the row
-    // of their queue entry.  The owner threads write chunk 6 (time features) and
-    // fence it, then each gather warp arrives on the slot's xfull barrier with the
-    // byte count its TMA gathers will deliver (expect_tx).
+  } else if (warp >= cs::BUILD_WARP0) {   // ============================ row builders
+    // Builder thread tb owns blocks tb and tb + 64 of each tile and computes, for every
+    // item (conv1 position j), the trace16 rows of their input rows 2j and 2j+1 and the
+    // time-feature chunks (cols 48..55: age, remaining-to-complete, remaining-to-retire of
+    // context rows, R2; zero otherwise) into the row ring, RQ items ahead of the TMA issue.
+    // Rows: padding -> the all-zero row past the rank's rows, R = 0 -> the current
+    // instruction, context rows newest first -> the row of queue entry k - R (R6).
     //
     // The metadata chain block id -> sub-trace state -> queue entries is staged in
     // shared memory by cp.async, one stage per tile or item ahead, so no register
@@ -375,45 +400,56 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // ids of tile t+3 and the states of tile t+2 (j == 0) and the queue entries of
     // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1:
     // one group per iteration).
-    const int m = tid - cs::GATHER_WARP0 * 32;
-    const int wq = warp - cs::GATHER_WARP0;          // gather warp 0..3: tile rows 32 wq .. 32 wq + 31
+    const int tb = (warp - cs::BUILD_WARP0) * 32 + lane;   // 0..63
     uint32_t* sIds = reinterpret_cast<uint32_t*>(sm + cs::SID_OFF);
     uint4* sMeta = reinterpret_cast<uint4*>(sm + cs::SMETA_OFF);
     uint4* sEnt = reinterpret_cast<uint4*>(sm + cs::SENT_OFF);
+    uint32_t* rRow = reinterpret_cast<uint32_t*>(sm + cs::RROW_OFF);
+    uint2* rT = reinterpret_cast<uint2*>(sm + cs::RT_OFF);
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const uint32_t n_items = my_tiles * 4;
-    auto valid_of = [&](uint32_t T) -> bool {         // block m of this CTA's T-th tile exists
+    auto valid_of = [&](uint32_t T, int m) -> bool {   // block m of this CTA's T-th tile exists
       const uint32_t tl = blockIdx.x + T * gridDim.x;
       return T < my_tiles && tl * cs::TILE + m < nblocks;
     };
-    auto stage_ids = [&](uint32_t T) {                // stage 1: block id of tile T
-      if (valid_of(T)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
-    };
-    auto stage_meta = [&](uint32_t T) {               // stage 2: sub-trace state of tile T (ids landed)
-      if (!valid_of(T)) return;
-      const uint32_t id = sIds[(T & 3) * 128 + m];
-      const uint32_t b = id >> 4;
-      uint4* d = sMeta + (T & 3) * 128 + m;
-      reinterpret_cast<uint32_t*>(d)[0] = id;
-      cp_async4(reinterpret_cast<uint32_t*>(d) + 1, a.count + b);
-      cp_async4(reinterpret_cast<uint32_t*>(d) + 2, a.ws + b);        // low word (little endian)
-      cp_async4(reinterpret_cast<uint32_t*>(d) + 3, a.clock + b);
-    };
-    auto stage_ent = [&](uint32_t n) {                // stage 3: queue entries of item n (states landed)
-      const uint32_t T = n >> 2;
-      if (!valid_of(T)) return;
-      const int j = (int)(n & 3);
-      const uint4 mt = sMeta[(T & 3) * 128 + m];
-      const int k = (int)mt.y;
+    auto stage_ids = [&](uint32_t T) {                 // stage 1: block ids of tile T
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int R = (int)(mt.x & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
-        if (R >= 1 && R <= k)                              // context row: entry k - R (newest first, R6)
-          cp_async16(sEnt + ((n & 3) * 128 + m) * 2 + h, a.q + (uint64_t)(k - R) * a.qn + (mt.x >> 4));
+      for (int u = 0; u < 2; ++u) {
+        const int m = tb + 64 * u;
+        if (valid_of(T, m)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
       }
     };
-    // One input row: the trace16 row the TMA fetches, and the time-feature chunk
-    // (cols 48..55) written next to it (context rows only, R2).
+    auto stage_meta = [&](uint32_t T) {                // stage 2: sub-trace states of tile T (ids landed)
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int m = tb + 64 * u;
+        if (!valid_of(T, m)) continue;
+        const uint32_t id = sIds[(T & 3) * 128 + m];
+        const uint32_t b = id >> 4;
+        uint32_t* d = reinterpret_cast<uint32_t*>(sMeta + (T & 3) * 128 + m);
+        d[0] = id;
+        cp_async4(d + 1, a.count + b);
+        cp_async4(d + 2, a.ws + b);        // low word (little endian)
+        cp_async4(d + 3, a.clock + b);
+      }
+    };
+    auto stage_ent = [&](uint32_t n) {                 // stage 3: queue entries of item n (states landed)
+      const uint32_t T = n >> 2;
+      const int j = (int)(n & 3);
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int m = tb + 64 * u;
+        if (!valid_of(T, m)) continue;
+        const uint4 mt = sMeta[(T & 3) * 128 + m];
+        const int k = (int)mt.y;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int R = (int)(mt.x & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
+          if (R >= 1 && R <= k)                              // context row: entry k - R (newest first, R6)
+            cp_async16(sEnt + ((n % 3) * 128 + m) * 2 + h, a.q + (uint64_t)(k - R) * a.qn + (mt.x >> 4));
+        }
+      }
+    };
     auto row_of = [&](bool valid, const uint4& mt, int R, const uint4& ev, uint2& tchunk) -> uint32_t {
       tchunk = make_uint2(0u, 0u);
       const int k = (int)mt.y;
@@ -425,11 +461,6 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
       return (uint32_t)((int64_t)ev.x - a.row_lo);
     };
-    // chunk 7 (cols 56..63) of every X row is never written by the TMA: zero it once
-#pragma unroll
-    for (int s2 = 0; s2 < cs::NX; ++s2)
-#pragma unroll
-      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
     // prologue: ids of tiles 0..2, states of tiles 0..1, entries of items 0..1
     for (uint32_t T = 0; T < 3; ++T) stage_ids(T);
     cp_async_commit();
@@ -445,49 +476,80 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;
       const int j = (int)(nI & 3);
+      if (warp == cs::BUILD_WARP0) PSIM_TS(112 + 3 * j);
       cp_async_wait<1>();                             // everything staged up to iteration nI - 2 has landed
-      if (j == 0 && warp == cs::GATHER_WARP0) PSIM_TS(80);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
-      const bool valid = valid_of(it);
-      const uint4 mt = sMeta[(it & 3) * 128 + m];
-      const uint4 e0 = sEnt[((nI & 3) * 128 + m) * 2], e1 = sEnt[((nI & 3) * 128 + m) * 2 + 1];
-      const int R0 = (int)(mt.x & 15) * 8 + 2 * j;
-      uint2 tA, tB;
-      const uint32_t rA = row_of(valid, mt, R0, e0, tA);
-      const uint32_t rB = row_of(valid, mt, R0 + 1, e1, tB);
-      const int xs = (int)(nI % cs::NX);
-      wait_empty(xempty + xs, nI / cs::NX);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
-      {
-        uint8_t* xa = sm + cs::X_OFF + xs * 32768;
-        // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
-        // writes only chunks 0..5, so this can go in before the rows land
-        st_sw128(xa, m, 6, make_uint4(tA.x, tA.y, 0u, 0u));
-        st_sw128(xa + 16384, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));
-        fence_async_smem();                               // chunk 6 visible to tcgen05
-        __syncwarp();
-        if (lane == 0) mbar_expect_tx(xfull + xs, 64 * 96);   // arrive + this warp's 64 rows of 96 B
-        __syncwarp();
-        // lane l < 16 fetches rows (atom h = l >> 3) of blocks 32 wq + 4 g .. + 3, g = l & 7
-        const int g = lane & 7, h = (lane >> 3) & 1;
-        uint32_t r4[4];
+      if (warp == cs::BUILD_WARP0) PSIM_TS(113 + 3 * j);
+      const int rs = (int)(nI % cs::RQ);
+      wait_empty(rempty + rs, nI / cs::RQ);
 #pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          const uint32_t va = __shfl_sync(0xffffffffu, rA, 4 * g + t);
-          const uint32_t vb = __shfl_sync(0xffffffffu, rB, 4 * g + t);
-          r4[t] = h ? vb : va;
-        }
-        if (lane < 16)
-          tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4[0], r4[1], r4[2], r4[3]);
+      for (int u = 0; u < 2; ++u) {
+        const int m = tb + 64 * u;
+        const bool valid = valid_of(it, m);
+        const uint4 mt = sMeta[(it & 3) * 128 + m];
+        const uint4 e0 = sEnt[((nI % 3) * 128 + m) * 2], e1 = sEnt[((nI % 3) * 128 + m) * 2 + 1];
+        const int R0 = (int)(mt.x & 15) * 8 + 2 * j;
+        uint2 tA, tB;
+        rRow[(rs * 2 + 0) * 128 + m] = row_of(valid, mt, R0, e0, tA);
+        rRow[(rs * 2 + 1) * 128 + m] = row_of(valid, mt, R0 + 1, e1, tB);
+        rT[(rs * 2 + 0) * 128 + m] = tA;
+        rT[(rs * 2 + 1) * 128 + m] = tB;
       }
-      if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(rfull + rs);
+      if (warp == cs::BUILD_WARP0) PSIM_TS(114 + 3 * j);
       // stage the metadata of later iterations
       if (j == 0) { stage_ids(it + 3); stage_meta(it + 2); }
       if (nI + 2 < n_items) stage_ent(nI + 2);
       cp_async_commit();
-      if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
     }
     cp_async_wait<0>();
+  } else if (warp >= cs::GATHER_WARP0) {   // ============================ TMA row issuers (warps 9..12)
+    // Operand row layout (per input row, 64 bf16): cols 0..46 the trace attributes,
+    // col 47 zero, cols 48..50 the time features, cols 51..63 zero.  The 96-B rows are
+    // fetched by the TMA unit with tile::gather4 (4 arbitrary trace16 rows per
+    // instruction, SWIZZLE_128B applied on the way) into chunks 0..5; thread m writes
+    // chunk 6 (time features) of its block's two rows, chunk 7 is zeroed once.  Each
+    // warp arrives on the slot's xfull barrier with the byte count its gathers deliver
+    // (expect_tx), so xfull completes when the last row lands.
+    const int m = tid - cs::GATHER_WARP0 * 32;
+    const int wq = warp - cs::GATHER_WARP0;          // issuer warp 0..3: tile rows 32 wq .. 32 wq + 31
+    const uint32_t* rRow = reinterpret_cast<const uint32_t*>(sm + cs::RROW_OFF);
+    const uint2* rT = reinterpret_cast<const uint2*>(sm + cs::RT_OFF);
+#pragma unroll
+    for (int s2 = 0; s2 < cs::NX; ++s2)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
+    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const uint32_t n_items = my_tiles * 4;
+    const int g = lane & 7, h = (lane >> 3) & 1;     // lane l < 16: rows of atom h, blocks 32 wq + 4 g .. + 3
+#pragma unroll 1
+    for (uint32_t nI = 0; nI < n_items; ++nI) {
+      const uint32_t it = nI >> 2;
+      const int j = (int)(nI & 3);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      const int rs = (int)(nI % cs::RQ);
+      wait_full(rfull + rs, nI / cs::RQ);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(104 + j);
+      const uint2 tA = rT[(rs * 2 + 0) * 128 + m], tB = rT[(rs * 2 + 1) * 128 + m];
+      const uint4 r4 = *reinterpret_cast<const uint4*>(rRow + (rs * 2 + h) * 128 + 32 * wq + 4 * g);
+      const int xs = (int)(nI % cs::NX);
+      wait_empty(xempty + xs, nI / cs::NX);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
+      uint8_t* xa = sm + cs::X_OFF + xs * 32768;
+      // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
+      // writes only chunks 0..5, so this can go in before the rows land
+      st_sw128(xa, m, 6, make_uint4(tA.x, tA.y, 0u, 0u));
+      st_sw128(xa + 16384, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));
+      fence_async_smem();                               // chunk 6 visible to tcgen05
+      __syncwarp();
+      if (lane == 0) mbar_expect_tx(xfull + xs, 64 * 96);   // arrive + this warp's 64 rows of 96 B
+      __syncwarp();
+      if (lane < 16)
+        tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(rempty + rs);          // ring slot consumed (its values are in registers)
+      if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
+    }
   }
   fence_before();
   __syncthreads();

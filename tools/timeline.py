@@ -23,7 +23,8 @@ for j in range(4):
     names[81 + 3 * j] = f"g{j}a"; names[82 + 3 * j] = f"g{j}slot"; names[83 + 3 * j] = f"g{j}xfull(prev)"
 for j in range(4):
     names[96 + 2 * j] = f"g{j}issued"; names[97 + 2 * j] = f"g{j}staged"
-    names[104 + 2 * j] = f"g{j}ownA"; names[105 + 2 * j] = f"g{j}ownB"
+    names[104 + j] = f"g{j}rfull"
+    names[112 + 3 * j] = f"b{j}top"; names[113 + 3 * j] = f"b{j}staged"; names[114 + 3 * j] = f"b{j}built"
 names.update({128: "tma start", 129: "tma end", 132: "mma wait tempty", 133: "mma start", 134: "mma issued",
               140: "epi start", 141: "epi F ready", 142: "epi y done", 145: "upd start", 146: "upd y ready",
               143: "upd done", 144: "upd scan"})
