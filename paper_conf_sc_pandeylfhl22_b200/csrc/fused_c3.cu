@@ -21,12 +21,12 @@
 // conv_stack_kernel roles (512 threads): warps 0..3 = EG-A (conv1 epilogue:
 // TMEM -> bias, ReLU, bf16 -> A2), warps 4..7 = EG-B (conv2 epilogue -> A3,
 // conv3 epilogue -> a4 rows, staged in smem and stored coalesced),
-// warp 8 = TMEM allocator, lane 0 the single-thread tcgen05.mma issuer;
+// warp 8 = TMEM allocator and MMA issuer (the whole warp runs the loop, one
+// elected lane issues; it also streams W3);
 // warps 9..12 = TMA row issuers (trace rows by tile::gather4 straight into the
 // SWIZZLE_128B X tile, time features from the row ring written by the
-// builders); warp 13 lane 0 = W3 streamer (its own warp: a spinning mbarrier
-// wait must never share a warp with the MMA issuer); warps 14..15 = row
-// builders (block id -> state -> queue entries -> row indices + time features).  W1/W2 stay
+// builders); warps 13..15 = row builders (block id -> state -> queue entries
+// -> row indices + time features).  W1/W2 stay
 // resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at a
 // time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
 // order is
@@ -66,10 +66,14 @@ static_assert(SMEM <= 232448, "conv_stack smem over the 227 KB opt-in limit");
 // 32 / 64 columns of the slot they were read from (packed bf16x2) and read by the MMA
 // from TMEM: no smem traffic for A2 / A3.
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;
-// warps 0-3 EG-A (conv1 epi), 4-7 EG-B (conv2/3 epi + a4 stores), 8 MMA, 9-12 TMA row
-// issuers, 13 W3 streamer, 14-15 row builders (metadata -> row indices + time features)
-constexpr int THREADS = 512;
-constexpr int MMA_WARP = 8, GATHER_WARP0 = 9, W3_WARP = 13, BUILD_WARP0 = 14;
+// warps 0-3 EG-A (conv1 epi + conv2 position 0 epi), 4-7 EG-B (conv2 position 1 + conv3
+// epi + a4 stores), 8 MMA + W3 stream, 9-11 row builders, 12-19 TMA row issuers (8 warps x
+// 8 lanes: the gather4 issue rate scales with issuing warps).  Five warpgroups; registers
+// rebalanced with setmaxnreg (each SM sub-partition holds one warp of every warpgroup):
+// EG-A 136 + EG-B 136 + MMA/builders 96 + issuers 56 + 56 = 480 <= 512.
+constexpr int THREADS = 640;
+constexpr int MMA_WARP = 8, BUILD_WARP0 = 9, NBUILD = 3, GATHER_WARP0 = 12, NISSUE = 8;
+constexpr int REG_EPI = 136, REG_ISSUE = 56;
 
 }  // namespace cs
 
@@ -128,6 +132,32 @@ __device__ void load_weight_sw128(uint8_t* dst, const __nv_bfloat16* w, int rows
   }
 }
 
+// conv2 epilogue of conv2 position h of a tile (one warp of a 4-warp epilogue group, TMEM
+// quadrant lane_base): C2 slot h (128 fp32) -> relu(+b2) -> bf16x2 written back into the
+// first 64 columns of the same slot (conv3's A operand), then a3full[h].
+__device__ __forceinline__ void conv2_epilogue(uint32_t tmem, uint32_t lane_base, const float* sb2, uint64_t* c2full,
+                                               uint64_t* a3full, uint32_t it, int h, int lane) {
+  wait_full(c2full + h, it);
+  fence_after();
+#pragma unroll 1
+  for (int cp = 0; cp < 2; ++cp) {   // channels 64 cp .. 64 cp + 63 -> A3 columns 32 cp .. 32 cp + 31
+    uint32_t r0[32], r1[32];
+    tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
+    tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
+    tmem_wait_ld();
+    uint32_t pk[32];
+    bias_relu_pack32(r0, sb2 + cp * 64, pk);
+    bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
+    // in place: columns 32 cp .. 32 cp + 31 were read already (cp = 1 reads 64 .. 127)
+    tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32, pk);
+    tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32 + 16, pk + 16);
+  }
+  tmem_wait_st();
+  fence_before();
+  __syncwarp();
+  if (lane == 0) mbar_arrive(a3full + h);
+}
+
 __global__ void __launch_bounds__(cs::THREADS, 1)
     conv_stack_kernel(ConvArgs a, const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2,
                       const __grid_constant__ CUtensorMap tmW3, const __grid_constant__ CUtensorMap tmX) {
@@ -154,8 +184,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (tid == 0) {
-    for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, 4); mbar_init(xempty + i, 1); }
-    for (int i = 0; i < cs::RQ; ++i) { mbar_init(rfull + i, 2); mbar_init(rempty + i, 4); }
+    for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, cs::NISSUE); mbar_init(xempty + i, 1); }
+    for (int i = 0; i < cs::RQ; ++i) { mbar_init(rfull + i, cs::NBUILD); mbar_init(rempty + i, cs::NISSUE); }
     for (int i = 0; i < 2; ++i) {
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 1); mbar_init(a2full + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 1); mbar_init(a3full + i, 4);
@@ -185,15 +215,32 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   const uint32_t nblocks = *a.nblocks;
   const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
   if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
-  if (warp < cs::GATHER_WARP0) mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
+  if (warp <= cs::MMA_WARP) mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
   const float* sb1 = reinterpret_cast<const float*>(sm + cs::BIAS_OFF);
   const float* sb2 = sb1 + 64;
   const float* sb3 = sb1 + 192;
 
   if (warp == cs::MMA_WARP) {
-    if (lane == 0) {   // ============================ MMA issuer
+    {   // ============================ MMA issuer
       // Per tile: c1(0) c1(1) [c3 of the previous tile, K-half 1] c2(0,*) c1(2) c1(3) c3(0) c2(1,*);
       // deferring the previous tile's last conv3 MMA lets this tile's conv1 overlap its epilogues.
+      // The whole warp runs this loop (descriptors stay warp-uniform, in uniform registers);
+      // one elected lane issues each MMA group and its commits.
+      const bool leader = elect_one();
+      // W3 stream (K-halves 0, 1, 0, 1, ... into one 32 KB buffer): fill f after the conv3
+      // MMAs of fill f-1 completed.  Issued two MMA groups ahead of its use, where that
+      // completion has normally already happened.
+      uint32_t nfill = 0;
+      auto fill = [&]() {
+        wait_empty(w3empty, nfill);
+        if (leader) {
+          mbar_expect_tx(w3full, 32 * 1024);
+          for (int a2 = 0; a2 < 2; ++a2)
+            tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (nfill & 1) + a2) * 64, 0);
+        }
+        __syncwarp();
+        ++nfill;
+      };
       const uint32_t sbase = smem_u32(sm);
       const uint32_t id64 = idesc_bf16(128, 64), id128 = idesc_bf16(128, 128);
       auto c1 = [&](uint32_t it, int j) {
@@ -206,12 +253,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         PSIM_TS(1 + 2 * j);
         fence_after();
         const uint32_t xa = sbase + cs::X_OFF + xs * 32768;
+        if (leader) {
 #pragma unroll
-        for (int k = 0; k < 8; ++k)
-          mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
-                   sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
-        mma_commit(xempty + xs);
-        mma_commit(c1full + s);
+          for (int k = 0; k < 8; ++k)
+            mma_bf16(tmem + cs::TMEM_C1 + s * 64, sw128_desc(xa + (k >> 2) * 16384 + (k & 3) * 32),
+                     sw128_desc(sbase + cs::W1_OFF + (k >> 2) * 8192 + (k & 3) * 32), id64, k > 0);
+          mma_commit(xempty + xs);
+          mma_commit(c1full + s);
+        }
+        __syncwarp();
       };
       auto c2 = [&](uint32_t it, int h, int kh) {   // conv2 position h, K-half kh = item 2h+kh (C1 slot kh)
         PSIM_TS(8 + 2 * (h * 2 + kh));
@@ -219,12 +269,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         if (kh == 0) wait_empty(c2empty + h, it);
         PSIM_TS(9 + 2 * (h * 2 + kh));
         fence_after();
+        if (leader) {
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
-          mma_bf16_ts(tmem + cs::TMEM_C2 + h * 128, tmem + cs::TMEM_C1 + kh * 64 + 8 * k,
-                      sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
-        mma_commit(c1empty + kh);   // C1 slot kh (its A2) free for conv1 two items later
-        if (kh == 1) mma_commit(c2full + h);
+          for (int k = 0; k < 4; ++k)
+            mma_bf16_ts(tmem + cs::TMEM_C2 + h * 128, tmem + cs::TMEM_C1 + kh * 64 + 8 * k,
+                        sw128_desc(sbase + cs::W2_OFF + kh * 16384 + k * 32), id128, (kh | k) != 0);
+          mma_commit(c1empty + kh);   // C1 slot kh (its A2) free for conv1 two items later
+          if (kh == 1) mma_commit(c2full + h);
+        }
+        __syncwarp();
       };
       auto c3 = [&](uint32_t it, int kh) {   // the (2 it + kh)-th conv3 MMA group: W3 K-half kh, A3 in C2 slot kh
         PSIM_TS(16 + 2 * kh);
@@ -233,24 +286,33 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         wait_full(w3full, it * 2 + kh);
         PSIM_TS(17 + 2 * kh);
         fence_after();
+        if (leader) {
 #pragma unroll
-        for (int k = 0; k < 8; ++k)
-          mma_bf16_ts(tmem + cs::TMEM_C3, tmem + cs::TMEM_C2 + kh * 128 + 8 * k,
-                      sw128_desc(sbase + cs::W3_OFF + (k >> 2) * 16384 + (k & 3) * 32), id128, (kh | k) != 0);
-        mma_commit(w3empty);
-        mma_commit(c2empty + kh);   // C2 slot kh free for the next tile's conv2 position kh
-        if (kh == 1) mma_commit(c3full);
+          for (int k = 0; k < 8; ++k)
+            mma_bf16_ts(tmem + cs::TMEM_C3, tmem + cs::TMEM_C2 + kh * 128 + 8 * k,
+                        sw128_desc(sbase + cs::W3_OFF + (k >> 2) * 16384 + (k & 3) * 32), id128, (kh | k) != 0);
+          mma_commit(w3empty);
+          mma_commit(c2empty + kh);   // C2 slot kh free for the next tile's conv2 position kh
+          if (kh == 1) mma_commit(c3full);
+        }
+        __syncwarp();
       };
       uint32_t it = 0;
       for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
+        if (it == 0) fill();                          // half 0 for c3(0, 0)
         c1(it, 0); c1(it, 1);
         if (it > 0) c3(it - 1, 1);
-        c2(it, 0, 0); c2(it, 0, 1); c1(it, 2); c1(it, 3); c3(it, 0); c2(it, 1, 0); c2(it, 1, 1);
+        c2(it, 0, 0); c2(it, 0, 1);
+        if (it > 0) fill();                           // half 0 for c3(it, 0): after c3(it - 1, 1)
+        c1(it, 2); c1(it, 3); c3(it, 0); c2(it, 1, 0);
+        fill();                                       // half 1 for c3(it, 1): after c3(it, 0)
+        c2(it, 1, 1);
       }
       if (it > 0) c3(it - 1, 1);
     }
     __syncwarp();
-  } else if (warp < 4) {   // ============================ EG-A: conv1 epilogues (C1 -> A2, in TMEM)
+  } else if (warp < 4) {   // ============ EG-A: conv1 epilogues (C1 -> A2, in TMEM) + conv2 position 0 epilogue
+    setmaxnreg_inc<cs::REG_EPI>();
     const int q = warp & 3;
     const int m = q * 32 + lane;                    // tile row = TMEM lane
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
@@ -281,39 +343,20 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(a2full + s);
         if (q == 0) PSIM_TS(48 + j);
+        if (j == 1) {   // conv2 position 0 (items 0 and 1) is complete after conv2 MMAs (0, *)
+          if (q == 0) PSIM_TS(56);
+          conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, 0, lane);
+          if (q == 0) PSIM_TS(59);
+        }
       }
     }
-  } else if (warp < 8) {   // ============================ EG-B: conv2 / conv3 epilogues
-    // Order per tile t: e2(t, 0), e3(t - 1), e2(t, 1).  e3(t - 1) becomes ready together
-    // with e2(t, 0) (conv3 K-half 1 of tile t-1 is issued just before conv2 of tile t);
-    // doing e2(t, 0) first lets conv3(t, 0) start while e3(t - 1) writes its rows out.
+  } else if (warp < 8) {   // ============================ EG-B: conv2 position 1 + conv3 epilogues
+    setmaxnreg_inc<cs::REG_EPI>();
+    // Order per tile t: e3(t - 1), then the conv2 epilogue of position 1 of tile t (position
+    // 0 is EG-A's, so conv3(t, 0) does not wait for e3(t - 1) to write its rows out).
     const int q = warp & 3;
     const int m = q * 32 + lane;
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
-    auto e2 = [&](uint32_t it, int h) {   // C2 slot h (128 fp32) -> relu(+b2) -> bf16 -> A3 (same slot)
-      if (q == 0) PSIM_TS(56 + 4 * h);
-      wait_full(c2full + h, it);
-      if (q == 0) PSIM_TS(57 + 4 * h);
-      fence_after();
-#pragma unroll 1
-      for (int cp = 0; cp < 2; ++cp) {   // channels 64 cp .. 64 cp + 63 -> A3 columns 32 cp .. 32 cp + 31
-        uint32_t r0[32], r1[32];
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 64 + 32, r1);
-        tmem_wait_ld();
-        uint32_t pk[32];
-        bias_relu_pack32(r0, sb2 + cp * 64, pk);
-        bias_relu_pack32(r1, sb2 + cp * 64 + 32, pk + 16);
-        // in place: columns 32 cp .. 32 cp + 31 were read already (cp = 1 reads 64 .. 127)
-        tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32, pk);
-        tmem_st16(tmem + lane_base + cs::TMEM_C2 + h * 128 + cp * 32 + 16, pk + 16);
-      }
-      tmem_wait_st();
-      fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(a3full + h);
-      if (q == 0) PSIM_TS(59 + 4 * h);
-    };
     // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p]: both halves are read out of TMEM first
     // (C3 released at once for the next tile's conv3), then one half row (64 channels,
     // 128 B) at a time is staged in this warp's 4 KB of the staging buffer (XOR-swizzled
@@ -367,27 +410,61 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     };
     uint32_t it = 0, prev_tl = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
-      e2(it, 0);
       if (it > 0) e3(it - 1, prev_tl);
-      e2(it, 1);
+      if (q == 0) PSIM_TS(60);
+      conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, 1, lane);
+      if (q == 0) PSIM_TS(63);
       prev_tl = tl;
     }
     if (it > 0) e3(it - 1, prev_tl);
-  } else if (warp == cs::W3_WARP) {
-    if (lane == 0) {   // ============================ W3 streamer
-      // conv3 MMA groups alternate K-halves 0, 1, 0, 1, ...; fill n waits until the
-      // MMAs of fill n-1 have finished reading the buffer, then loads half n & 1
-      uint32_t nfill = 0;
-      for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) nfill += 2;
-      for (uint32_t f = 0; f < nfill; ++f) {
-        wait_empty(w3empty, f);
-        mbar_expect_tx(w3full, 32 * 1024);
-        for (int a2 = 0; a2 < 2; ++a2)
-          tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, (int)(2 * (f & 1) + a2) * 64, 0);
-      }
+  } else if (warp >= cs::GATHER_WARP0) {   // ============================ TMA row issuers (warps 12..19)
+    // Operand row layout (per input row, 64 bf16): cols 0..46 the trace attributes,
+    // col 47 zero, cols 48..50 the time features, cols 51..63 zero.  The 96-B rows are
+    // fetched by the TMA unit with tile::gather4 (4 arbitrary trace16 rows per
+    // instruction, SWIZZLE_128B applied on the way) into chunks 0..5: issuer warp wq
+    // covers blocks 16 wq .. 16 wq + 15 (lanes 0..7: gather4 of blocks 16 wq + 4 g .. + 3,
+    // atom h); lane l writes chunk 6 (time features) of block 16 wq + (l & 15), atom l >> 4;
+    // chunk 7 is zeroed once.  Each warp arrives on the slot's xfull barrier with the byte
+    // count its gathers deliver (expect_tx), so xfull completes when the last row lands.
+    setmaxnreg_dec<cs::REG_ISSUE>();
+    const int wq = warp - cs::GATHER_WARP0;          // issuer warp 0..7
+    const int m = 16 * wq + (lane & 15), hh = lane >> 4;
+    const uint32_t* rRow = reinterpret_cast<const uint32_t*>(sm + cs::RROW_OFF);
+    const uint2* rT = reinterpret_cast<const uint2*>(sm + cs::RT_OFF);
+#pragma unroll
+    for (int s2 = 0; s2 < cs::NX; ++s2) st_sw128(sm + cs::X_OFF + s2 * 32768 + hh * 16384, m, 7, make_uint4(0, 0, 0, 0));
+    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const uint32_t n_items = my_tiles * 4;
+    const int g = lane & 3, h = (lane >> 2) & 1;     // lane l < 8: rows of atom h, blocks 16 wq + 4 g .. + 3
+#pragma unroll 1
+    for (uint32_t nI = 0; nI < n_items; ++nI) {
+      const uint32_t it = nI >> 2;   // tile (timestamps only)
+      const int j = (int)(nI & 3);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      const int rs = (int)(nI % cs::RQ);
+      wait_full(rfull + rs, nI / cs::RQ);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(104 + j);
+      const uint2 tc = rT[(rs * 2 + hh) * 128 + m];
+      const uint4 r4 = *reinterpret_cast<const uint4*>(rRow + (rs * 2 + h) * 128 + 16 * wq + 4 * g);
+      const int xs = (int)(nI % cs::NX);
+      wait_empty(xempty + xs, nI / cs::NX);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
+      uint8_t* xa = sm + cs::X_OFF + xs * 32768;
+      // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
+      // writes only chunks 0..5, so this can go in before the rows land
+      st_sw128(xa + hh * 16384, m, 6, make_uint4(tc.x, tc.y, 0u, 0u));
+      fence_async_smem();                               // chunk 6 visible to tcgen05
+      __syncwarp();
+      if (lane == 0) mbar_expect_tx(xfull + xs, 32 * 96);   // arrive + this warp's 32 rows of 96 B
+      __syncwarp();
+      if (lane < 8)
+        tma_gather4(xa + h * 16384 + (16 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(rempty + rs);          // ring slot consumed (its values are in registers)
+      if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
     }
-  } else if (warp >= cs::BUILD_WARP0) {   // ============================ row builders
-    // Builder thread tb owns blocks tb and tb + 64 of each tile and computes, for every
+  } else {   // ============================ row builders (warps 9..11)
+    // Builder thread tb owns blocks tb and tb + 96 (< 128) of each tile and computes, for every
     // item (conv1 position j), the trace16 rows of their input rows 2j and 2j+1 and the
     // time-feature chunks (cols 48..55: age, remaining-to-complete, remaining-to-retire of
     // context rows, R2; zero otherwise) into the row ring, RQ items ahead of the TMA issue.
@@ -400,7 +477,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // ids of tile t+3 and the states of tile t+2 (j == 0) and the queue entries of
     // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1:
     // one group per iteration).
-    const int tb = (warp - cs::BUILD_WARP0) * 32 + lane;   // 0..63
+    const int tb = (warp - cs::BUILD_WARP0) * 32 + lane;   // 0..95: blocks tb and tb + 96 (< 128)
+    constexpr int NB = cs::NBUILD * 32;
     uint32_t* sIds = reinterpret_cast<uint32_t*>(sm + cs::SID_OFF);
     uint4* sMeta = reinterpret_cast<uint4*>(sm + cs::SMETA_OFF);
     uint4* sEnt = reinterpret_cast<uint4*>(sm + cs::SENT_OFF);
@@ -415,15 +493,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     auto stage_ids = [&](uint32_t T) {                 // stage 1: block ids of tile T
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
-        const int m = tb + 64 * u;
-        if (valid_of(T, m)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
+        const int m = tb + NB * u;
+        if (m < cs::TILE && valid_of(T, m)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
       }
     };
     auto stage_meta = [&](uint32_t T) {                // stage 2: sub-trace states of tile T (ids landed)
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
-        const int m = tb + 64 * u;
-        if (!valid_of(T, m)) continue;
+        const int m = tb + NB * u;
+        if (m >= cs::TILE || !valid_of(T, m)) continue;
         const uint32_t id = sIds[(T & 3) * 128 + m];
         const uint32_t b = id >> 4;
         uint32_t* d = reinterpret_cast<uint32_t*>(sMeta + (T & 3) * 128 + m);
@@ -438,8 +516,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       const int j = (int)(n & 3);
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
-        const int m = tb + 64 * u;
-        if (!valid_of(T, m)) continue;
+        const int m = tb + NB * u;
+        if (m >= cs::TILE || !valid_of(T, m)) continue;
         const uint4 mt = sMeta[(T & 3) * 128 + m];
         const int k = (int)mt.y;
 #pragma unroll
@@ -483,7 +561,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       wait_empty(rempty + rs, nI / cs::RQ);
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
-        const int m = tb + 64 * u;
+        const int m = tb + NB * u;
+        if (m >= cs::TILE) continue;
         const bool valid = valid_of(it, m);
         const uint4 mt = sMeta[(it & 3) * 128 + m];
         const uint4 e0 = sEnt[((nI % 3) * 128 + m) * 2], e1 = sEnt[((nI % 3) * 128 + m) * 2 + 1];
@@ -503,53 +582,6 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       cp_async_commit();
     }
     cp_async_wait<0>();
-  } else if (warp >= cs::GATHER_WARP0) {   // ============================ TMA row issuers (warps 9..12)
-    // Operand row layout (per input row, 64 bf16): cols 0..46 the trace attributes,
-    // col 47 zero, cols 48..50 the time features, cols 51..63 zero.  The 96-B rows are
-    // fetched by the TMA unit with tile::gather4 (4 arbitrary trace16 rows per
-    // instruction, SWIZZLE_128B applied on the way) into chunks 0..5; thread m writes
-    // chunk 6 (time features) of its block's two rows, chunk 7 is zeroed once.  Each
-    // warp arrives on the slot's xfull barrier with the byte count its gathers deliver
-    // (expect_tx), so xfull completes when the last row lands.
-    const int m = tid - cs::GATHER_WARP0 * 32;
-    const int wq = warp - cs::GATHER_WARP0;          // issuer warp 0..3: tile rows 32 wq .. 32 wq + 31
-    const uint32_t* rRow = reinterpret_cast<const uint32_t*>(sm + cs::RROW_OFF);
-    const uint2* rT = reinterpret_cast<const uint2*>(sm + cs::RT_OFF);
-#pragma unroll
-    for (int s2 = 0; s2 < cs::NX; ++s2)
-#pragma unroll
-      for (int h = 0; h < 2; ++h) st_sw128(sm + cs::X_OFF + s2 * 32768 + h * 16384, m, 7, make_uint4(0, 0, 0, 0));
-    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    const uint32_t n_items = my_tiles * 4;
-    const int g = lane & 7, h = (lane >> 3) & 1;     // lane l < 16: rows of atom h, blocks 32 wq + 4 g .. + 3
-#pragma unroll 1
-    for (uint32_t nI = 0; nI < n_items; ++nI) {
-      const uint32_t it = nI >> 2;
-      const int j = (int)(nI & 3);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
-      const int rs = (int)(nI % cs::RQ);
-      wait_full(rfull + rs, nI / cs::RQ);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(104 + j);
-      const uint2 tA = rT[(rs * 2 + 0) * 128 + m], tB = rT[(rs * 2 + 1) * 128 + m];
-      const uint4 r4 = *reinterpret_cast<const uint4*>(rRow + (rs * 2 + h) * 128 + 32 * wq + 4 * g);
-      const int xs = (int)(nI % cs::NX);
-      wait_empty(xempty + xs, nI / cs::NX);
-      if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
-      uint8_t* xa = sm + cs::X_OFF + xs * 32768;
-      // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
-      // writes only chunks 0..5, so this can go in before the rows land
-      st_sw128(xa, m, 6, make_uint4(tA.x, tA.y, 0u, 0u));
-      st_sw128(xa + 16384, m, 6, make_uint4(tB.x, tB.y, 0u, 0u));
-      fence_async_smem();                               // chunk 6 visible to tcgen05
-      __syncwarp();
-      if (lane == 0) mbar_expect_tx(xfull + xs, 64 * 96);   // arrive + this warp's 64 rows of 96 B
-      __syncwarp();
-      if (lane < 16)
-        tma_gather4(xa + h * 16384 + (32 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w);
-      __syncwarp();
-      if (lane == 0) mbar_arrive(rempty + rs);          // ring slot consumed (its values are in registers)
-      if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
-    }
   }
   fence_before();
   __syncthreads();

@@ -205,6 +205,18 @@ __device__ __forceinline__ void bias_relu_pack32(const uint32_t (&r)[32], const 
 }
 // 16-byte store into a K-major SWIZZLE_128B tile: row m (128 B), logical
 // 16-byte chunk c (0..7) lands in physical chunk c ^ (m & 7).
+// one elected lane of a converged warp (the MMA / TMA issue idiom: the whole warp runs
+// the issue loop so its operands stay warp-uniform, one lane issues)
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred;
+  asm volatile("{\n.reg .pred P;\nelect.sync _|P, 0xffffffff;\nselp.u32 %0, 1, 0, P;\n}\n" : "=r"(pred));
+  return pred != 0;
+}
+// warpgroup register rebalancing (all 4 warps of a warpgroup execute the same one)
+template <int N>
+__device__ __forceinline__ void setmaxnreg_dec() { asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N)); }
+template <int N>
+__device__ __forceinline__ void setmaxnreg_inc() { asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N)); }
 __device__ __forceinline__ void st_sw128(uint8_t* atom, int m, int c, uint4 v) {
   *reinterpret_cast<uint4*>(atom + m * 128 + ((c ^ (m & 7)) << 4)) = v;
 }
