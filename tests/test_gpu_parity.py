@@ -351,3 +351,25 @@ def test_trace_residency_modes_identical(chunk):
             assert st["trace_mode"] == {"device": 0, "pinned": 1, "pageable": 2}[mode]
     assert totals[0] == totals[1] == totals[2]
     assert np.array_equal(cycles[0], cycles[1]) and np.array_equal(cycles[0], cycles[2])
+
+
+def test_fused_deterministic_many_tiles():
+    """Race detector for the fused path: with several 128-block tiles per CTA per step
+    (every pipeline buffer of conv_stack / fc1_head wraps many times), repeated runs and
+    the pinned streaming mode give bit-identical per-sub-trace cycles.  (An early version
+    of the conv3 staging buffer that a neighbouring warp could overwrite passed every
+    single-tile test and failed exactly this.)"""
+    L, N, W = 480_000, 40_000, 24
+    tr = synth.trace(L, 777)
+    w = synth.weights("C3")
+    pinned = torch.from_numpy(tr).pin_memory()
+    runs = []
+    for src in ("device", "device", "pinned"):
+        with P.Simulator(precision="bf16") as sim:
+            sim.load_trace(torch.from_numpy(tr).cuda() if src == "device" else pinned)
+            sim.partition(N, W)
+            sim.load_model("C3", w)
+            sim.simulate()
+            runs.append((sim.total_cycles(), sim.subtrace_cycles()))
+    for t, c in runs[1:]:
+        assert t == runs[0][0] and np.array_equal(c, runs[0][1])
