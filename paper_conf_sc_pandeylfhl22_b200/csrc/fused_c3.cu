@@ -1098,7 +1098,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   a.ws = g.ws; a.clock = g.clock; a.count = g.count;
   a.q = g.q;
   a.step = step;
-  a.qn = g.n;
+  a.qn = g.qn ? g.qn : g.n;
   a.w1 = f.w1; a.w2 = f.w2; a.w3 = f.w3;
   a.b1 = f.b1; a.b2 = f.b2; a.b3 = f.b3;
   a.a4 = f.a4;

@@ -54,6 +54,8 @@ struct Model {
 // Per-rank lockstep state: structure-of-arrays in HBM, sub-trace-major.
 struct SimState {
   uint64_t n = 0;               // local sub-traces
+  uint64_t qn = 0;              // queue entry stride (0: n); a cohort's view of a larger state keeps
+                                // the full state's stride (its pointers are offset by its first sub-trace)
   int64_t* ws = nullptr;        // [n] first row (warm-up start)
   int64_t* s = nullptr;         // [n] first real row
   int64_t* e = nullptr;         // [n] end row
@@ -95,6 +97,7 @@ struct GatherArgs {
   uint64_t n;
   int64_t step;
   int item_rows = kRows;     // rows per sub-trace in x (RB7: 116)
+  uint64_t qn = 0;           // queue entry stride (0: n)
   int row_off = 0;           // row of the current instruction inside an item (RB7: 2)
 };
 void launch_gather_f32(const GatherArgs& a, float* x, cudaStream_t st);

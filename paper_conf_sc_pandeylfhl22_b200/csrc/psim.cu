@@ -82,6 +82,7 @@ struct Prof {
     if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
     return pool[used++];
   }
+  void count(int cls) { launches[cls]++; }
   void begin(int cls) {
     launches[cls]++;
     if (!on || !sample) return;
@@ -108,10 +109,26 @@ struct Prof {
   ~Prof() { for (auto e : pool) cudaEventDestroy(e); }
 };
 
+// A cohort: a contiguous block of this rank's sub-traces simulated on its own stream
+// with its own fused-path block lists, so the kernels of different cohorts overlap on
+// the device (one cohort's conv_stack fills the SMs another cohort's fc1_head tail and
+// the kernel boundaries leave idle).  Sub-traces are independent, so the
+// results are bit-identical to one cohort.
+struct Cohort {
+  FusedC3 fz;                 // shared model/trace fields + this cohort's per-run buffers
+  cudaStream_t st = nullptr;
+  cudaEvent_t ev = nullptr;
+  uint64_t b0 = 0, n = 0, cap = 0;
+  uint32_t* blocks = nullptr;
+  uint32_t* count = nullptr;
+  uint8_t* tileP[2] = {nullptr, nullptr};
+};
+
 struct psim_ctx {
   psim_opts opts{};
   Prof prof;
   FusedC3 fused;
+  std::vector<Cohort> cohorts;
   int cap = 110;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -253,6 +270,11 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->fused.tileP[0]);
   dfree(ctx->fused.tileP[1]);
   dfree(ctx->fused.a4);
+  for (Cohort& c : ctx->cohorts) {
+    dfree(c.blocks); dfree(c.count); dfree(c.tileP[0]); dfree(c.tileP[1]);
+    if (c.st) cudaStreamDestroy(c.st);
+    if (c.ev) cudaEventDestroy(c.ev);
+  }
   for (void* p : {(void*)ctx->pec.k1, (void*)ctx->pec.c1, (void*)ctx->pec.ws, (void*)ctx->pec.s, (void*)ctx->pec.e,
                   (void*)ctx->pec.bnd, (void*)ctx->pec.cyc, (void*)ctx->pec.cycles1, (void*)ctx->pec.len,
                   (void*)ctx->pec.corrected, (void*)ctx->pec.rec_lat, (void*)ctx->pec.rec_k})
@@ -853,6 +875,51 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     launch_fused_init(ctx->fused, n, st);
     pf.end(PSIM_KC_OTHER);
   }
+  // cohorts (fused first pass without correction / interval metrics): PSIM_COHORTS, default
+  // 2 when the trace streams from pinned host memory (measured on config 3: e2e 406 -> 428
+  // MIPS, the chunk copies overlap better), 1 otherwise (device-resident: 537.6 vs 537.0,
+  // 3-4 cohorts slower; profiles/r01_cohorts.txt)
+  int ncoh = 1;
+  if (fused && n && !pec && !metrics) {
+    const char* ev = getenv("PSIM_COHORTS");
+    ncoh = ev ? std::max(1, atoi(ev)) : (stream_load ? 2 : 1);
+    while (ncoh > 1 && n < (uint64_t)ncoh * 256) --ncoh;
+  }
+  if (ncoh > 1) {
+    if ((int)ctx->cohorts.size() < ncoh) ctx->cohorts.resize(ncoh);
+    CK(cudaEventRecord(ctx->ev[3], st));   // common preparation done
+    for (int c = 0; c < ncoh; ++c) {
+      Cohort& ch = ctx->cohorts[c];
+      const uint64_t b0 = (n * (uint64_t)c / ncoh) & ~uint64_t(127), b1 = c + 1 == ncoh ? n : (n * (uint64_t)(c + 1) / ncoh) & ~uint64_t(127);
+      ch.b0 = b0; ch.n = b1 - b0;
+      if (!ch.st) CK(cudaStreamCreateWithFlags(&ch.st, cudaStreamNonBlocking));
+      if (!ch.ev) CK(cudaEventCreateWithFlags(&ch.ev, cudaEventDisableTiming));
+      if (ch.cap < ch.n) {
+        dfree(ch.blocks); dfree(ch.count); dfree(ch.tileP[0]); dfree(ch.tileP[1]);
+        const uint64_t nt = (ch.n + 127) / 128;
+        CK(cudaMalloc(&ch.blocks, ch.n * 14 * 4));
+        CK(cudaMalloc(&ch.count, 16));
+        CK(cudaMalloc(&ch.tileP[0], nt + 16));
+        CK(cudaMalloc(&ch.tileP[1], nt + 16));
+        ch.cap = ch.n;
+      }
+      ch.fz = ctx->fused;
+      ch.fz.blocks = ch.blocks; ch.fz.count = ch.count; ch.fz.tileP[0] = ch.tileP[0]; ch.fz.tileP[1] = ch.tileP[1];
+      ch.fz.a4 = ctx->fused.a4 + b0 * 14 * 128;
+      if (!fused_make_maps(ch.fz, ch.n)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for a cohort");
+      CK(cudaStreamWaitEvent(ch.st, ctx->ev[3], 0));
+      launch_fused_init(ch.fz, ch.n, ch.st);
+      pf.count(PSIM_KC_OTHER);
+    }
+  }
+  // a cohort's view of the state: pointers offset by its first sub-trace, queue stride kept
+  auto view = [&](const SimState& s0, uint64_t b0, uint64_t nc) {
+    SimState v = s0;
+    v.n = nc; v.qn = s0.n;
+    v.ws = s0.ws + b0; v.s = s0.s + b0; v.e = s0.e + b0; v.clock = s0.clock + b0; v.bnd = s0.bnd + b0;
+    v.cycles = s0.cycles + b0; v.count = s0.count + b0; v.rmin = s0.rmin + b0; v.q = s0.q + b0;
+    return v;
+  };
   // one lockstep step t of a pass: gather -> CNN -> rounding -> queue update
   auto step = [&](GatherArgs& g, UpdateArgs& u, const int64_t* e_arr, int64_t t) -> int {
     if (fused) {
@@ -881,11 +948,47 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     pf.end(PSIM_KC_UPDATE);
     return PSIM_OK;
   };
-  for (int64_t t = 0; t < ctx->steps && n; ++t) {
-    if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
-    pf.sample = t % Prof::kEvery == 0;
-    rc = step(ga, ua, ctx->st.e, t);
-    if (rc) return rc;
+  if (ncoh > 1) {
+    // cohorts on their own streams, launches interleaved step by step; cohort 0's
+    // launches carry the (sampled) kernel timing, the others are counted only
+    std::vector<GatherArgs> gc(ncoh, ga);
+    std::vector<UpdateArgs> uc(ncoh, ua);
+    for (int c = 0; c < ncoh; ++c) {
+      const Cohort& ch = ctx->cohorts[c];
+      const SimState v = view(ctx->st, ch.b0, ch.n);
+      gc[c].ws = v.ws; gc[c].e = v.e; gc[c].clock = v.clock; gc[c].count = v.count; gc[c].q = v.q;
+      gc[c].n = ch.n; gc[c].qn = n;
+      uc[c].st = v;
+    }
+    cudaStream_t st0 = pf.st;
+    for (int64_t t = 0; t < ctx->steps; ++t) {
+      for (int c = 0; c < ncoh; ++c) {
+        Cohort& ch = ctx->cohorts[c];
+        if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(ch.st, ctx->ld_events[t / chunk], 0));
+        gc[c].step = t; uc[c].step = t;
+        const bool timed = c == 0 && t % Prof::kEvery == 0;
+        pf.st = ch.st;
+        pf.sample = timed;
+        pf.begin(PSIM_KC_LAYER0);
+        launch_conv_stack(ch.fz, gc[c], t, ch.n, ch.st);
+        pf.end(PSIM_KC_LAYER0);
+        pf.begin(PSIM_KC_LAYER0 + 3);
+        launch_fc1_head(ch.fz, uc[c], ctx->st.e + ch.b0, t, forced, ch.st);
+        pf.end(PSIM_KC_LAYER0 + 3);
+      }
+    }
+    pf.st = st0;
+    for (int c = 0; c < ncoh; ++c) {
+      CK(cudaEventRecord(ctx->cohorts[c].ev, ctx->cohorts[c].st));
+      CK(cudaStreamWaitEvent(st, ctx->cohorts[c].ev, 0));
+    }
+  } else {
+    for (int64_t t = 0; t < ctx->steps && n; ++t) {
+      if (stream_load && t % chunk == 0) CK(cudaStreamWaitEvent(st, ctx->ld_events[t / chunk], 0));
+      pf.sample = t % Prof::kEvery == 0;
+      rc = step(ga, ua, ctx->st.e, t);
+      if (rc) return rc;
+    }
   }
   pf.sample = true;
   // ---- post-error correction pass (PAPER.md:203-219 [V-B], Fig. 9; R19) ----

@@ -90,7 +90,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
   }
   int64_t clock = a.st.clock[b];
   const int k = a.st.count[b];
-  const uint64_t qn = a.st.n;                            // entry stride (entry-major layout)
+  const uint64_t qn = a.st.qn ? a.st.qn : a.st.n;        // entry stride (entry-major layout)
   uint4* qb = a.st.q + b;
   const uint32_t code = a.mrow ? a.mrow[i - a.row_lo] : 0u;   // metrics tag of row i (R20)
   const uint32_t clo_before = (uint32_t)clock;
@@ -179,7 +179,7 @@ struct QBatch { uint32_t s[8], f[8], c[8], w[8]; };
 
 // first 8 entries of sub-trace b (entry-major layout), to be prefetched early
 __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int k, QBatch& q) {
-  const uint64_t qn = st.n;
+  const uint64_t qn = st.qn ? st.qn : st.n;
 #pragma unroll
   for (int t = 0; t < 8; ++t)
     if (t < k) { const uint4 v = st.q[t * qn + b]; q.s[t] = v.x; q.f[t] = v.y; q.c[t] = v.z; q.w[t] = v.w; }
@@ -200,7 +200,7 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
   } else {
     f = pf; c = pc; s = ps;
   }
-  const uint64_t qn = a.st.n;                              // entry-major: entry e at [e * n + b]
+  const uint64_t qn = a.st.qn ? a.st.qn : a.st.n;          // entry-major: entry e at [e * qn + b]
   uint4* qb = a.st.q + b;
   const uint32_t code = a.mrow ? a.mrow[i - a.row_lo] : 0u;   // metrics tag of row i (R20)
   const uint32_t clo_before = (uint32_t)clock;
