@@ -202,6 +202,9 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     bulk_g2s(sbias + 192, a.b3, 512, wbar);
     for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W1_OFF + kc * 8192, &tmW1, wbar, kc * 64, 0);
     for (int kc = 0; kc < 2; ++kc) tma_load_2d(sm + cs::W2_OFF + kc * 16384, &tmW2, wbar, kc * 64, 0);
+    // W3 fill 0 (K-half 0 for the first tile's conv3) also before the PDL wait
+    mbar_expect_tx(w3full, 32 * 1024);
+    for (int a2 = 0; a2 < 2; ++a2) tma_load_2d(sm + cs::W3_OFF + a2 * 16384, &tmW3, w3full, a2 * 64, 0);
   }
   if (warp == cs::MMA_WARP) tmem_alloc(tmem_slot, cs::TMEM_COLS);
   fence_before();
@@ -230,7 +233,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       // W3 stream (K-halves 0, 1, 0, 1, ... into one 32 KB buffer): fill f after the conv3
       // MMAs of fill f-1 completed.  Issued two MMA groups ahead of its use, where that
       // completion has normally already happened.
-      uint32_t nfill = 0;
+      uint32_t nfill = 1;   // fill 0 was issued with the resident weights, before the PDL wait
       auto fill = [&]() {
         wait_empty(w3empty, nfill);
         if (leader) {
@@ -299,7 +302,6 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       };
       uint32_t it = 0;
       for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
-        if (it == 0) fill();                          // half 0 for c3(0, 0)
         c1(it, 0); c1(it, 1);
         if (it > 0) c3(it - 1, 1);
         c2(it, 0, 0); c2(it, 0, 1);
@@ -309,6 +311,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         c2(it, 1, 1);
       }
       if (it > 0) c3(it - 1, 1);
+      if (it == 0) wait_full(w3full, 0);   // no tile: still let fill 0 land before the CTA exits
     }
     __syncwarp();
   } else if (warp < 4) {   // ============ EG-A: conv1 epilogues (C1 -> A2, in TMEM) + conv2 position 0 epilogue
@@ -667,9 +670,24 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
-  grid_dep_wait();                 // PDL: a4, block counts and queue state of conv_stack / the previous step
+  // PDL: every role waits (griddepcontrol.wait) for a4, block counts and queue state of
+  // conv_stack / the previous step before touching them; the TMA producer first puts the
+  // weight (B) halves of its first tile's first stages in flight: W_fc1 does not depend on
+  // the previous kernels, and tileP of this step was written by the previous fc1_head,
+  // complete before conv_stack of this step passed its own wait (and so before this
+  // kernel could launch).
   grid_dep_launch_dependents();
   const bool run_head = (a.u.forced == nullptr) || a.force_predict;
+  int npre = 0;   // producer: k-blocks of the first tile whose B half was issued before the wait
+  if (warp == 0 && lane == 0 && run_head && blockIdx.x < ntiles) {
+    npre = min(2 * (int)a.tileP[blockIdx.x], fh::STAGES);
+    for (int kb = 0; kb < npre; ++kb) {
+      uint8_t* sa = sm + kb * fh::STAGE;
+      mbar_expect_tx(full + kb, fh::STAGE);
+      tma_load_2d(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0);
+    }
+  }
+  grid_dep_wait();
   if (warp >= 2 && warp < 6) mbar_wait(cbar, 0);   // epilogue warps read T and fc2 from smem
 
   if (warp == 0) {
@@ -680,11 +698,15 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         const int nk = 2 * a.tileP[tt];
         PSIM_TS(128);
         for (int kb = 0; kb < nk; ++kb) {
-          mbar_wait(empty + stage, phase ^ 1);
           uint8_t* sa = sm + stage * fh::STAGE;
-          mbar_expect_tx(full + stage, fh::STAGE);
-          tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
-          tma_load_2d(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0);
+          if (it == 0 && kb < npre) {                 // B already in flight (issued before the PDL wait)
+            tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
+          } else {
+            mbar_wait(empty + stage, phase ^ 1);
+            mbar_expect_tx(full + stage, fh::STAGE);
+            tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
+            tma_load_2d(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0);
+          }
           if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
         }
         PSIM_TS(129);
