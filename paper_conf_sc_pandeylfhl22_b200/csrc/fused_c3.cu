@@ -439,6 +439,10 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const uint32_t n_items = my_tiles * 4;
     const int g = lane & 3, h = (lane >> 2) & 1;     // lane l < 8: rows of atom h, blocks 16 wq + 4 g .. + 3
+    // trace rows are streamed through L2 with evict_first (PSIM_ROW_EVICT=0: normal): the
+    // step's context rows (~145 MB at config 3, G = 1) exceed L2 and would otherwise push
+    // out the queue entries, states and a4 rows that are reused within the step
+    const uint64_t pol = l2_policy_evict_first();
 #pragma unroll 1
     for (uint32_t nI = 0; nI < n_items; ++nI) {
       const uint32_t it = nI >> 2;   // tile (timestamps only)
@@ -461,7 +465,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (lane == 0) mbar_expect_tx(xfull + xs, 32 * 96);   // arrive + this warp's 32 rows of 96 B
       __syncwarp();
       if (lane < 8)
-        tma_gather4(xa + h * 16384 + (16 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w);
+        tma_gather4_hint(xa + h * 16384 + (16 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w, pol);
       __syncwarp();
       if (lane == 0) mbar_arrive(rempty + rs);          // ring slot consumed (its values are in registers)
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
