@@ -688,7 +688,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     for (int kb = 0; kb < npre; ++kb) {
       uint8_t* sa = sm + kb * fh::STAGE;
       mbar_expect_tx(full + kb, fh::STAGE);
-      tma_load_2d(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0);
+      tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0, l2_policy_evict_last());
     }
   }
   grid_dep_wait();
@@ -696,6 +696,8 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
 
   if (warp == 0) {
     if (lane == 0 && run_head) {   // ---- TMA producer
+      // L2 policies: a4 rows are read once per step (evict_first), W_fc1 by every tile (evict_last)
+      const uint64_t polA = l2_policy_evict_first(), polB = l2_policy_evict_last();
       uint32_t stage = 0, phase = 0;
       uint32_t it = 0;
       for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
@@ -704,12 +706,12 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         for (int kb = 0; kb < nk; ++kb) {
           uint8_t* sa = sm + stage * fh::STAGE;
           if (it == 0 && kb < npre) {                 // B already in flight (issued before the PDL wait)
-            tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
+            tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
           } else {
             mbar_wait(empty + stage, phase ^ 1);
             mbar_expect_tx(full + stage, fh::STAGE);
-            tma_load_2d(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM));
-            tma_load_2d(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0);
+            tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
+            tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0, polB);
           }
           if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
         }
