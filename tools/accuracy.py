@@ -63,14 +63,14 @@ def config4(a):
     10M-instruction trace; error against the same GPU simulator at N = 1 (the unpartitioned
     CPU oracle would need ~1e14 FLOP single-threaded; the GPU path agrees with it to ~1e-5
     on the S3 parity cases)."""
-    L = 10_000_000
+    L = a.L if a.L != 200_000 else 10_000_000
     seed = synth.TRACE_SEED_BASE + 4
     tr = synth.trace(L, seed)
     w = synth.weights("C3")
     ref, _, t_ref = run(tr, 1, 0, 0, w)
     print(f"unpartitioned: total {ref} in {t_ref:.1f} s", flush=True)
     rows = []
-    for N in [256 << i for i in range(11)]:
+    for N in [256 << i for i in range(11) if (256 << i) * 8 <= L]:
         for W in (0, 128, 1000, 10000):
             tot, _, t = run(tr, N, W, 0, w)
             rows.append(dict(N=N, W=W, total=tot, err=(tot - ref) / ref, seconds=t))
