@@ -51,8 +51,7 @@ constexpr int NX = 3;                        // X slots: gathered items in fligh
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
 constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][128 B] (half rows)
 // gather metadata staged by cp.async (no register waits on loads in flight):
-constexpr int SID_OFF = STG_OFF + 16 * 1024; // u32   [4 tiles][128]    block ids
-constexpr int SMETA_OFF = SID_OFF + 2048;    // uint4 [4 tiles][128]    {id, k, ws lo, Clock lo}
+constexpr int SMETA_OFF = STG_OFF + 16 * 1024;   // uint4 [4 tiles][128] block entries {id, k, ws lo, Clock lo}
 constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [3 items][128][2] queue entries of rows 2j, 2j+1 (item n in slot n % 3)
 constexpr int RQ = 3;                        // row ring: items built ahead of the TMA issue
 constexpr int RROW_OFF = SENT_OFF + 3 * 4096; // u32   [RQ][2][128] trace16 row of input row 2j+h of block m
@@ -78,7 +77,7 @@ constexpr int REG_EPI = 136, REG_ISSUE = 56;
 }  // namespace cs
 
 struct ConvArgs {
-  const uint32_t* blocks;    // block ids (b << 4 | p) of this step
+  const uint4* blocks;       // block entries {b << 4 | p, k, ws lo, Clock lo} of this step
   const uint32_t* nblocks;   // count of this step's list
   uint32_t* next_count;      // the other step parity's counter, reset here
   const __nv_bfloat16* trace16;   // [rows + 1][48] bf16 operand rows (attributes at cols 0..46), row `rows` zero
@@ -366,7 +365,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // by 16-B chunk) and written out coalesced: one instruction stores four 128-B half rows.
     auto e3 = [&](uint32_t it, uint32_t tl) {
       const uint32_t bi = tl * cs::TILE + m;
-      const uint32_t id = bi < nblocks ? a.blocks[bi] : 0xFFFFFFFFu;
+      const uint32_t id = bi < nblocks ? a.blocks[bi].x : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
       wait_full(c3full, it);                          // conv3 accumulated
       if (q == 0) PSIM_TS(65);
@@ -478,15 +477,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // Rows: padding -> the all-zero row past the rank's rows, R = 0 -> the current
     // instruction, context rows newest first -> the row of queue entry k - R (R6).
     //
-    // The metadata chain block id -> sub-trace state -> queue entries is staged in
-    // shared memory by cp.async, one stage per tile or item ahead, so no register
-    // ever waits on a load in flight: iteration n (tile t, item j) issues the block
-    // ids of tile t+3 and the states of tile t+2 (j == 0) and the queue entries of
-    // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1:
-    // one group per iteration).
+    // The metadata chain block entry (id + the sub-trace state, written with the id by
+    // the previous step's update) -> queue entries is staged in shared memory by
+    // cp.async, so no register ever waits on a load in flight: iteration n (tile t,
+    // item j) issues the block entries of tile t+2 (j == 0) and the queue entries of
+    // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1: one
+    // group per iteration).
     const int tb = (warp - cs::BUILD_WARP0) * 32 + lane;   // 0..95: blocks tb and tb + 96 (< 128)
     constexpr int NB = cs::NBUILD * 32;
-    uint32_t* sIds = reinterpret_cast<uint32_t*>(sm + cs::SID_OFF);
     uint4* sMeta = reinterpret_cast<uint4*>(sm + cs::SMETA_OFF);
     uint4* sEnt = reinterpret_cast<uint4*>(sm + cs::SENT_OFF);
     uint32_t* rRow = reinterpret_cast<uint32_t*>(sm + cs::RROW_OFF);
@@ -497,28 +495,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       const uint32_t tl = blockIdx.x + T * gridDim.x;
       return T < my_tiles && tl * cs::TILE + m < nblocks;
     };
-    auto stage_ids = [&](uint32_t T) {                 // stage 1: block ids of tile T
+    auto stage_meta = [&](uint32_t T) {                // stage 1: block entries {id, k, ws lo, Clock lo} of tile T
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
         const int m = tb + NB * u;
-        if (m < cs::TILE && valid_of(T, m)) cp_async4(sIds + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
+        if (m < cs::TILE && valid_of(T, m))
+          cp_async16(sMeta + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
       }
     };
-    auto stage_meta = [&](uint32_t T) {                // stage 2: sub-trace states of tile T (ids landed)
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int m = tb + NB * u;
-        if (m >= cs::TILE || !valid_of(T, m)) continue;
-        const uint32_t id = sIds[(T & 3) * 128 + m];
-        const uint32_t b = id >> 4;
-        uint32_t* d = reinterpret_cast<uint32_t*>(sMeta + (T & 3) * 128 + m);
-        d[0] = id;
-        cp_async4(d + 1, a.count + b);
-        cp_async4(d + 2, a.ws + b);        // low word (little endian)
-        cp_async4(d + 3, a.clock + b);
-      }
-    };
-    auto stage_ent = [&](uint32_t n) {                 // stage 3: queue entries of item n (states landed)
+    auto stage_ent = [&](uint32_t n) {                 // stage 2: queue entries of item n (block entries landed)
       const uint32_t T = n >> 2;
       const int j = (int)(n & 3);
 #pragma unroll
@@ -546,10 +531,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
       return (uint32_t)((int64_t)ev.x - a.row_lo);
     };
-    // prologue: ids of tiles 0..2, states of tiles 0..1, entries of items 0..1
-    for (uint32_t T = 0; T < 3; ++T) stage_ids(T);
-    cp_async_commit();
-    cp_async_wait<0>();
+    // prologue: block entries of tiles 0..1, queue entries of items 0..1
     for (uint32_t T = 0; T < 2; ++T) stage_meta(T);
     cp_async_commit();
     cp_async_wait<0>();
@@ -584,7 +566,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       if (lane == 0) mbar_arrive(rfull + rs);
       if (warp == cs::BUILD_WARP0) PSIM_TS(114 + 3 * j);
       // stage the metadata of later iterations
-      if (j == 0) { stage_ids(it + 3); stage_meta(it + 2); }
+      if (j == 0) stage_meta(it + 2);
       if (nI + 2 < n_items) stage_ent(nI + 2);
       cp_async_commit();
     }
@@ -623,7 +605,7 @@ struct HeadArgs {
   const int64_t* e;
   const uint8_t* tileP;      // [ntiles] P_tile of this step
   uint8_t* tileP_next;       // [ntiles] P_tile of the next step
-  uint32_t* blocks_next;     // block list of the next step
+  uint4* blocks_next;        // block list of the next step
   uint32_t* next_count;
   __nv_bfloat16* a4;         // [n][14][128] (zero-fill of [P_b, P_tile) for the next step)
   const float* T;            // [15][256] constant table
@@ -836,13 +818,14 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const float y0 = yrow[0], y1 = yrow[1], y2 = yrow[2];
       __syncwarp();
       if (lane == 0) mbar_arrive(yempty + yb);
-      int pnext = 0;
+      int pnext = 0, knext = 0;
       if (active) {
         bool stopped = false;
         const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, rmin, first, run_head, y0, y1, y2, sHist,
                                                 &stopped);
         if (a.u.step + 1 < nsteps && !stopped) {
           pnext = (knew + 8) >> 3;                 // ceil((k+1)/8)
+          knext = knew;
           // keep a4 rows >= P_b zero: clear the rows this sub-trace no longer computes
           for (int p = pnext; p < pb; ++p) {
             uint4* dst = reinterpret_cast<uint4*>(a.a4 + (b * 14 + p) * 128);
@@ -876,7 +859,8 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       named_bar_sync(2 + grp, 128);
       const uint32_t base = (uint32_t)sPg[8] + (uint32_t)(before + incl - pnext);
       if (q == 0) PSIM_TS(144);
-      for (int p = 0; p < pnext; ++p) a.blocks_next[base + p] = (uint32_t)(b << 4) | (uint32_t)p;
+      for (int p = 0; p < pnext; ++p)
+        a.blocks_next[base + p] = make_uint4((uint32_t)(b << 4) | (uint32_t)p, (uint32_t)knext, (uint32_t)ws, (uint32_t)clock);
       named_bar_sync(2 + grp, 128);   // sP reused by the next tile
     }
   }
@@ -976,9 +960,10 @@ void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64
 }
 
 // step-0 block list: every sub-trace has k = 0 -> P = 1
-__global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count, uint8_t* tileP, uint32_t* next_count) {
+__global__ void fused_init_kernel(uint64_t n, const int64_t* __restrict__ ws, uint4* blocks, uint32_t* count,
+                                  uint8_t* tileP, uint32_t* next_count) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (t < n) blocks[t] = (uint32_t)(t << 4);
+  if (t < n) blocks[t] = make_uint4((uint32_t)(t << 4), 0u, (uint32_t)ws[t], 0u);   // empty queue, Clock 0
   if (t < (n + 127) / 128) tileP[t] = 1;
   if (t == 0) { *count = (uint32_t)n; *next_count = 0; }
 }
@@ -986,8 +971,9 @@ __global__ void fused_init_kernel(uint64_t n, uint32_t* blocks, uint32_t* count,
 // step-0 block list of a pass that starts from existing queues (correction pass):
 // one CTA of 128 threads per 128-sub-trace tile, P_b = ceil((k+1)/8) for active b
 __global__ void __launch_bounds__(128) fused_init_state_kernel(uint64_t n, const int32_t* __restrict__ count,
+                                                                const int64_t* __restrict__ clock,
                                                                 const int64_t* __restrict__ ws,
-                                                                const int64_t* __restrict__ e, uint32_t* blocks,
+                                                                const int64_t* __restrict__ e, uint4* blocks,
                                                                 uint32_t* nblocks, uint8_t* tileP) {
   __shared__ int sSum[4], sMax[4], sBase;
   const int m = threadIdx.x, lane = m & 31, w = m >> 5;
@@ -1014,14 +1000,15 @@ __global__ void __launch_bounds__(128) fused_init_state_kernel(uint64_t n, const
   int before = 0;
   for (int q = 0; q < w; ++q) before += sSum[q];
   const uint32_t base = (uint32_t)sBase + (uint32_t)(before + incl - P);
-  for (int p = 0; p < P; ++p) blocks[base + p] = (uint32_t)(b << 4) | (uint32_t)p;
+  for (int p = 0; p < P; ++p)
+    blocks[base + p] = make_uint4((uint32_t)(b << 4) | (uint32_t)p, (uint32_t)count[b], (uint32_t)ws[b], (uint32_t)clock[b]);
 }
 
-void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* ws, const int64_t* e,
+void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* clock, const int64_t* ws, const int64_t* e,
                                   uint64_t n, cudaStream_t st) {
   cudaMemsetAsync(f.count, 0, 8, st);
   const uint64_t nt = (n + 127) / 128;
-  if (nt) fused_init_state_kernel<<<(unsigned)nt, 128, 0, st>>>(n, count, ws, e, f.blocks, f.count, f.tileP[0]);
+  if (nt) fused_init_state_kernel<<<(unsigned)nt, 128, 0, st>>>(n, count, clock, ws, e, f.blocks, f.count, f.tileP[0]);
 }
 
 // ---------------------------------------------------------------- host side
@@ -1080,9 +1067,9 @@ static void launch_pdl(void (*kern)(KArgs...), int grid, int threads, int smem, 
   cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
-void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st) {
+void launch_fused_init(FusedC3& f, const int64_t* ws, uint64_t n, cudaStream_t st) {
   const uint64_t th = n > 1 ? n : 1;
-  fused_init_kernel<<<(unsigned)((th + 255) / 256), 256, 0, st>>>(n, f.blocks, f.count + 0, f.tileP[0], f.count + 1);
+  fused_init_kernel<<<(unsigned)((th + 255) / 256), 256, 0, st>>>(n, ws, f.blocks, f.count + 0, f.tileP[0], f.count + 1);
 }
 
 // PSIM_DEBUG_TIMING=<step>: CTA 0 of conv_stack records clock64() at every

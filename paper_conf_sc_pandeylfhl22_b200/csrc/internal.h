@@ -195,7 +195,8 @@ struct FusedC3 {
   const float* head_b = nullptr;
   // per-run buffers (owned), sized for cap_n sub-traces
   uint64_t cap_n = 0;
-  uint32_t* blocks = nullptr;         // [n*14] block ids b<<4|p
+  uint4* blocks = nullptr;            // [n*14] block entries {b<<4|p, k_b, ws_b lo, Clock_b lo}: the sub-trace
+                                      // state the gather needs travels with the block id (one 16-B read)
   uint32_t* count = nullptr;          // [2] block counts by step parity
   uint8_t* tileP[2] = {nullptr, nullptr};   // [ceil(n/128)] P_tile by step parity
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
@@ -204,10 +205,10 @@ struct FusedC3 {
   CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][48] (box 48 x 1, SWIZZLE_128B)
   uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)
 };
-void launch_fused_init(FusedC3& f, uint64_t n, cudaStream_t st);
+void launch_fused_init(FusedC3& f, const int64_t* ws, uint64_t n, cudaStream_t st);
 // block list / P_tile of step 0 of a pass whose sub-traces start from a non-empty
 // queue (the correction pass): P_b = ceil((count+1)/8) for active b (ws < e)
-void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* ws, const int64_t* e,
+void launch_fused_init_from_state(FusedC3& f, const int32_t* count, const int64_t* clock, const int64_t* ws, const int64_t* e,
                                   uint64_t n, cudaStream_t st);
 // trace rows (uint8 attributes) -> bf16 operand rows of the fused conv1 layout
 void launch_trace16(const uint8_t* trace, int64_t stride, int64_t rows, __nv_bfloat16* out, cudaStream_t st);

@@ -119,7 +119,7 @@ struct Cohort {
   cudaStream_t st = nullptr;
   cudaEvent_t ev = nullptr;
   uint64_t b0 = 0, n = 0, cap = 0;
-  uint32_t* blocks = nullptr;
+  uint4* blocks = nullptr;
   uint32_t* count = nullptr;
   uint8_t* tileP[2] = {nullptr, nullptr};
 };
@@ -734,7 +734,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       dfree(fz.blocks); dfree(fz.count); dfree(fz.tileP[0]); dfree(fz.tileP[1]); dfree(fz.a4);
       fz.blocks = nullptr; fz.count = nullptr; fz.tileP[0] = fz.tileP[1] = nullptr; fz.a4 = nullptr;
       const uint64_t nt = (nn + 127) / 128;
-      CK(cudaMalloc(&fz.blocks, nn * 14 * 4));
+      CK(cudaMalloc(&fz.blocks, nn * 14 * 16));
       CK(cudaMalloc(&fz.count, 16));
       CK(cudaMalloc(&fz.tileP[0], nt + 16));
       CK(cudaMalloc(&fz.tileP[1], nt + 16));
@@ -872,7 +872,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     // invariant of the fused path: a4 rows p >= P_b are zero (fc1 reads them as 0)
     CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
     pf.begin(PSIM_KC_OTHER);
-    launch_fused_init(ctx->fused, n, st);
+    launch_fused_init(ctx->fused, ctx->st.ws, n, st);
     pf.end(PSIM_KC_OTHER);
   }
   // cohorts (fused first pass without correction / interval metrics): PSIM_COHORTS, default
@@ -897,7 +897,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       if (ch.cap < ch.n) {
         dfree(ch.blocks); dfree(ch.count); dfree(ch.tileP[0]); dfree(ch.tileP[1]);
         const uint64_t nt = (ch.n + 127) / 128;
-        CK(cudaMalloc(&ch.blocks, ch.n * 14 * 4));
+        CK(cudaMalloc(&ch.blocks, ch.n * 14 * 16));
         CK(cudaMalloc(&ch.count, 16));
         CK(cudaMalloc(&ch.tileP[0], nt + 16));
         CK(cudaMalloc(&ch.tileP[1], nt + 16));
@@ -908,7 +908,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       ch.fz.a4 = ctx->fused.a4 + b0 * 14 * 128;
       if (!fused_make_maps(ch.fz, ch.n)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for a cohort");
       CK(cudaStreamWaitEvent(ch.st, ctx->ev[3], 0));
-      launch_fused_init(ch.fz, ch.n, ch.st);
+      launch_fused_init(ch.fz, ctx->st.ws + ch.b0, ch.n, ch.st);
       pf.count(PSIM_KC_OTHER);
     }
   }
@@ -1021,7 +1021,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       // a4 rows >= P_b must be zero again: the final steps of the first pass leave rows behind
       CK(cudaMemsetAsync(ctx->fused.a4, 0, n * 14 * 128 * 2, st));
       pf.begin(PSIM_KC_OTHER);
-      launch_fused_init_from_state(ctx->fused, ctx->st.count, p.ws, p.e, n, st);
+      launch_fused_init_from_state(ctx->fused, ctx->st.count, ctx->st.clock, p.ws, p.e, n, st);
       pf.end(PSIM_KC_OTHER);
     }
     for (int64_t t = 0; t < p.limit; ++t) {

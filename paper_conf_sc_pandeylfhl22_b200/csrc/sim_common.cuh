@@ -186,7 +186,7 @@ __device__ __forceinline__ void load_qbatch(const SimState& st, uint64_t b, int 
 }
 
 __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint64_t b, int64_t ws, int64_t s_b,
-                                                      int64_t nsteps, int k, int64_t clock, uint32_t rmin,
+                                                      int64_t nsteps, int k, int64_t& clock, uint32_t rmin,
                                                       const QBatch& first, bool has_y, float y0, float y1, float y2,
                                                       unsigned int* hist, bool* stopped = nullptr) {
   const int64_t i = ws + a.step;
