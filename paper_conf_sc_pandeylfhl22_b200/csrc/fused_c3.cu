@@ -18,17 +18,17 @@
 // folded into T[P] = b_fc1 + sum_{p >= P} Wfc1[:, p] c3 (R18).
 // P_b = ceil((k_b + 1) / 8).  Exact in real arithmetic; the oracle stays dense.
 //
-// conv_stack_kernel roles (512 threads): warps 0..3 = EG-A (conv1 epilogue:
-// TMEM -> bias, ReLU, bf16 -> A2), warps 4..7 = EG-B (conv2 epilogue -> A3,
-// conv3 epilogue -> a4 rows, staged in smem and stored coalesced),
-// warp 8 = TMEM allocator and MMA issuer (the whole warp runs the loop, one
-// elected lane issues; it also streams W3);
-// warps 9..12 = TMA row issuers (trace rows by tile::gather4 straight into the
-// SWIZZLE_128B X tile, time features from the row ring written by the
-// builders); warps 13..15 = row builders (block id -> state -> queue entries
-// -> row indices + time features).  W1/W2 stay
-// resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at a
-// time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
+// conv_stack_kernel roles (640 threads, five warpgroups, registers rebalanced with
+// setmaxnreg): warps 0..3 = EG-A (conv1 epilogue: TMEM -> bias, ReLU, bf16 -> A2 back
+// into TMEM, and the epilogue of conv2 position 0), warps 4..7 = EG-B (conv2
+// position 1 -> A3 in TMEM, conv3 epilogue -> a4 rows, staged in smem and stored
+// coalesced), warp 8 = TMEM allocator and MMA issuer (the whole warp runs the loop,
+// one elected lane issues; it also streams W3), warps 9..11 = row builders (block
+// entry {id, k, ws, Clock} -> queue entries -> row indices + time features, staged
+// by cp.async), warps 12..19 = TMA row issuers (trace rows by tile::gather4 straight
+// into the SWIZZLE_128B X tile, evict_first; time features from the row ring).
+// W1/W2 stay resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at
+// a time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
 // order is
 //   c1(0) c1(1) [c3(prev,1)] c2(0,0) c2(0,1) c1(2) c1(3) c3(0) c2(1,0) c2(1,1)
 // with K-split accumulation; the conv2 / conv3 A operands live in TMEM.
