@@ -953,7 +953,16 @@ void launch_load_chunk16(const uint8_t* host_rows, int64_t host_first_row, int64
                          const int64_t* e, uint64_t n, int64_t t0, int64_t t1, int64_t row_lo,
                          __nv_bfloat16* trace16, uint8_t* mrow, cudaStream_t st) {
   uint64_t blocks = (n * 32 + 127) / 128;
-  if (blocks > 148ull * 2) blocks = 148ull * 2;   // ~one 4-warp CTA per SM next to the compute kernels
+  // Loader grid cap (PSIM_LOADER_CTAS, default 64): each loader CTA takes an SM slot the
+  // fused kernels need at every kernel boundary, so fewer, longer-lived loader CTAs slow
+  // the simulation far less while still streaming faster than it consumes rows --
+  // measured on config 3 (2 cohorts): e2e 446 / 476 / 533 / 528 / 500 MIPS with
+  // 296 / 32 / 64 / 48 / 128 CTAs (tools/gpu/loaderctas.sh)
+  static const uint64_t cap = [] {
+    const char* e = getenv("PSIM_LOADER_CTAS");
+    return (uint64_t)(e && atoi(e) > 0 ? atoi(e) : 64);
+  }();
+  if (blocks > cap) blocks = cap;
   if (blocks < 1) blocks = 1;
   load_chunk16_kernel<<<(unsigned)blocks, 128, 0, st>>>(host_rows, host_first_row, stride, ws, e, n, t0, t1, row_lo,
                                                          trace16, mrow);
