@@ -4,8 +4,10 @@
 
 Compiles every csrc/*.cu with ``-gencode arch=compute_100a,code=sm_100a
 -lineinfo -O3`` (cross-compiles on a CPU-only box) and links one shared
-library with the CUDA runtime linked statically, so the .so that travels to
-the GPU box is self-contained.  NCCL is resolved at run time with dlopen.
+library against the shared CUDA runtime (libcudart.so.12, rpath
+/usr/local/cuda/lib64, present in the same image on the GPU box; when torch
+is imported first its already-loaded libcudart.so.12 is reused).  NCCL is
+resolved at run time with dlopen.
 """
 from __future__ import annotations
 
@@ -65,7 +67,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
         objs = list(ex.map(compile_one, _sources()))
     tmp = LIB + f".{os.getpid()}.tmp"
-    cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-ldl", "-lpthread"]
+    cmd = [NVCC] + ARCH + ["-shared", "-cudart", "shared", "-Xlinker", "-rpath,/usr/local/cuda/lib64",
+                          "-o", tmp] + objs + ["-ldl", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
