@@ -72,7 +72,7 @@ class ClockSampler:
         q = "index,clocks.sm,clocks.max.sm,power.draw," + ",".join(f"clocks_event_reasons.{r}" for r in REASONS)
         try:
             self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
-                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL, start_new_session=True)
+                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL, start_new_session=True)
         except FileNotFoundError:
             self.p = None
 
@@ -103,6 +103,21 @@ def peaks():
 
 
 # --------------------------------------------------------------------------- roofline
+# Algorithmic FLOP of the fused C3 path (SURVEY.md §8(d) "full constant-folding" count,
+# DESIGN.md §5), per block (sub-trace b, conv3 position p < P_b) and per sub-trace:
+CONV1_FLOP = 4 * 2 * 100 * 64      # 4 conv1 positions per block; K = 2 taps x 50 real features
+CONV2_FLOP = 2 * 2 * 128 * 128     # 2 conv2 positions; K = 2 taps x 64 channels
+CONV3_FLOP = 2 * 256 * 128         # 1 conv3 position; K = 2 taps x 128 channels
+CONV_STACK_FLOP_PER_BLOCK = CONV1_FLOP + CONV2_FLOP + CONV3_FLOP   # 182,272
+FC1_FLOP_PER_BLOCK = 2 * 128 * 256  # fc1 over the P_b computed positions (x 128 channels)
+FC2_FLOP_PER_SUBTRACE = 2 * 256 * 3
+
+
+def step_flops(blocks_per_step, n_active):
+    """Algorithmic FLOP of one lockstep step: 247,808 per block + 1,536 per sub-trace."""
+    return blocks_per_step * (CONV_STACK_FLOP_PER_BLOCK + FC1_FLOP_PER_BLOCK) + n_active * FC2_FLOP_PER_SUBTRACE
+
+
 def roofline(stats, k_steps, cfg):
     """Dominant kernel class by device time; algorithmic work per launch / average
     launch duration (CUDA events on the launch stream, PSIM_PROFILE)."""
@@ -115,6 +130,7 @@ def roofline(stats, k_steps, cfg):
     hist = np.array(stats["k_hist"], np.float64)
     kmean = float((hist * np.arange(112)).sum() / max(hist.sum(), 1))
     fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0   # fused path: conv_stack + fc1_head
+    sustained = pk["bf16_tflops_sustained"]
     if cfg["arch"] == "RB7" and names[dom].startswith("gemm_layer"):
         # layer-wise tcgen05 GEMMs, reported together (one kernel, 8 launches per step): stem
         # 2*56*100*64 + six k3 convs 6 * 2*56*192*64 + fc1 2*3584*256 per simulated instruction
@@ -122,26 +138,27 @@ def roofline(stats, k_steps, cfg):
         g_ms = sum(ms[i] for i in g)
         flops = float(stats["simulated"]) * k_steps * (716800 + 6 * 1376256 + 1835008)
         achieved = flops / (g_ms / 1e3) / 1e12
-        peak = pk["bf16_tflops_sustained"]
         out.update(kernel="gemm_tc_kernel (all RB7 layers)", share=round(g_ms / total_ms, 4), bound="tensor",
-                   achieved=round(achieved, 2), peak=peak, unit="TFLOP/s", frac=round(achieved / peak, 4),
-                   flops_per_step=flops / k_steps, peak_source=src + " bf16 sustained")
+                   achieved=round(achieved, 2), peak=sustained, unit="TFLOP/s", frac=round(achieved / sustained, 4),
+                   flops_per_step=flops / k_steps, peak_source=src + " bf16_tflops_sustained")
         avg_s = g_ms / 1e3 / max(sum(launches[i] for i in g), 1)
     elif names[dom].startswith("gemm_layer"):
         li = int(names[dom][-1])
         M, N, K = stats["layer_m"][li], stats["layer_n"][li], stats["layer_k"][li]
-        if fused and li == 0:     # conv_stack: per (sub-trace, position) block conv1 4x2x100x64 + conv2 2x2x128x128 + conv3 2x256x128
-            flops = float(M) * 247808.0
-        elif fused and li == 3:   # fc1 over P_tile positions (tile max of P_b): K = 128 * mean P_tile
-            flops = 2.0 * M * 256 * (stats["layer_k"][3] / 1000.0)
+        if fused and li == 0:     # conv_stack: M = mean blocks per step (= per launch)
+            flops = float(M) * CONV_STACK_FLOP_PER_BLOCK
+        elif fused and li == 3:   # fc1_head: fc1 over the P_b computed positions of each sub-trace + fc2
+            flops = float(stats["layer_m"][0]) * FC1_FLOP_PER_BLOCK + float(M) * FC2_FLOP_PER_SUBTRACE
         else:
             k_alg = 100 if li == 0 else K      # conv1: 2 rows x 50 real features (features padded to 64)
             flops = 2.0 * M * N * k_alg
         achieved = flops / avg_s / 1e12
-        peak = pk["bf16_tflops_sustained"] if cfg["precision"] == "bf16" else 74.0
+        peak = sustained if cfg["precision"] == "bf16" else 74.0
         out.update(bound="tensor", achieved=round(achieved, 2), peak=peak, unit="TFLOP/s",
                    frac=round(achieved / peak, 4), flops_per_launch=flops,
-                   peak_source=(src + " bf16 sustained") if cfg["precision"] == "bf16" else "derived fp32 SIMT")
+                   flops_per_unit=(CONV_STACK_FLOP_PER_BLOCK if (fused and li == 0) else None),
+                   unit_of_work=("block (sub-trace, conv3 position p < P_b)" if (fused and li == 0) else None),
+                   peak_source=(src + " bf16_tflops_sustained") if cfg["precision"] == "bf16" else "derived fp32 SIMT")
     else:
         n = stats["subtraces"]
         if names[dom] == "gather":   # X write (bf16 112x64) + trace rows (k+1)x48 + queue (k x 12 B)
@@ -156,6 +173,15 @@ def roofline(stats, k_steps, cfg):
     if fused:
         out["kernel"] = {"gemm_layer0": "conv_stack_kernel (gather+conv1+conv2+conv3, fused)",
                          "gemm_layer3": "fc1_head_kernel (fc1+head+update, fused)"}.get(names[dom], names[dom])
+        # whole lockstep step: all algorithmic FLOP of the step / mean step time (sim_ms / steps)
+        bps = float(stats["layer_m"][0])
+        n_act = float(stats["simulated"]) / max(stats["steps"], 1)
+        fl = step_flops(bps, n_act)
+        step_s = stats["sim_ms"] / 1e3 / max(stats["steps"], 1)
+        out["step"] = {"flops": fl, "ms": round(step_s * 1e3, 5), "achieved": round(fl / step_s / 1e12, 2),
+                       "frac": round(fl / step_s / 1e12 / sustained, 4), "blocks": round(bps, 1),
+                       "note": "algorithmic FLOP of a mean lockstep step (247,808 per block + 1,536 per active "
+                               "sub-trace) / (simulate device time / steps), whole simulate incl. reduction"}
     out["kernels"] = {names[i]: {"ms": round(ms[i] / k_steps, 3), "launches": launches[i] // k_steps,
                                  "share": round(ms[i] / total_ms, 4) if total_ms else None}
                       for i in range(len(names)) if launches[i]}
@@ -173,14 +199,14 @@ def ncu_traffic(kernel_class):
 
 
 # --------------------------------------------------------------------------- CPU oracle
-def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None):
+def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None, seed=7):
     """Run the oracle (as it stands, single thread) on whole sub-traces of the same
     workload until ~budget_s of CPU time; returns (instructions, seconds, cycles)."""
     import oracle
     import synth
     w = synth.weights(cfg["arch"])
     mode = oracle.BF16 if cfg["precision"] == "bf16" else oracle.FP64
-    rng = np.random.default_rng(7)
+    rng = np.random.default_rng(seed)
     done, t_used, per = 0, 0.0, {}
     js = list(j_list) if j_list is not None else []
     while True:
@@ -207,6 +233,45 @@ def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None):
     return done, t_used, per
 
 
+def _oracle_worker(args):
+    """One all-core oracle process: whole random sub-traces for ~budget_s of its own CPU."""
+    cfg_name, budget_s, seed = args
+    cfg = CONFIGS[cfg_name]
+    os.environ.setdefault("OMP_NUM_THREADS", "1")
+    n_i, t, per = oracle_sample(cfg, None, 0, budget_s, cfg["L"], cfg["N"], cfg["W"], seed=seed)
+    return n_i, t, len(per)
+
+
+def host_info():
+    info = {"nproc": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        keep = ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core", "CPU(s)", "CPU max MHz")
+        for ln in out.splitlines():
+            k, _, v = ln.partition(":")
+            if k.strip() in keep:
+                info["lscpu " + k.strip()] = v.strip()
+    except Exception as ex:  # noqa: BLE001 - informational only
+        info["lscpu"] = f"unavailable: {ex}"
+    return info
+
+
+def oracle_all_cores(cfg_name, budget_s):
+    """The oracle as it stands on every host core: P = nproc independent processes, each
+    simulating whole random sub-traces of the same workload for ~budget_s.  Returns
+    (instructions, wall seconds, P, sub-traces)."""
+    import multiprocessing as mp
+    P = host_info()["nproc"]
+    ctx = mp.get_context("spawn")
+    t0 = time.perf_counter()
+    with ctx.Pool(P) as pool:
+        res = pool.map(_oracle_worker, [(cfg_name, budget_s, 1000 + i) for i in range(P)])
+    wall = time.perf_counter() - t0
+    # per-process throughput is measured on its own clock; aggregate = sum of per-process rates
+    rate = sum(n / t for n, t, _ in res if t > 0)
+    return sum(n for n, _, _ in res), wall, P, sum(c for _, _, c in res), rate
+
+
 # --------------------------------------------------------------------------- main
 def main():
     ap = argparse.ArgumentParser()
@@ -215,7 +280,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="psim", choices=["psim", "reference"])
     ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
-    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of single-thread oracle work for cpu_baseline")
+    ap.add_argument("--cpu-budget-all", type=float, default=12.0,
+                    help="seconds per process of the all-core oracle run (P = nproc processes)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg (profiling runs)")
     ap.add_argument("--emulate-rank", default=None, metavar="R/G",
@@ -227,8 +294,20 @@ def main():
     cfg = CONFIGS[args.config]
     L, N, W = cfg["L"], cfg["N"], cfg["W"]
 
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # started without torchrun: launch one rank per GPU ourselves (same arguments)
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        log("[bench] launching", " ".join(cmd))
+        sys.exit(subprocess.call(cmd))
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus and args.impl != "reference":
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch one rank per GPU")
     emu = None
     if args.emulate_rank:
         emu = tuple(int(x) for x in args.emulate_rank.split("/"))   # (R, G): partition as rank R of G
@@ -242,22 +321,32 @@ def main():
         # the oracle as it stands, on rank 0 only, on the host cores
         if rank != 0:
             return
-        import synth  # noqa: F401
-        per_step = max(2.0, args.cpu_budget / 3)
-        times, insts = [], 0
-        for it in range(args.warmup + args.steps):
-            n_i, t, _ = oracle_sample(cfg, None, 0, per_step, L, N, W)
-            if it >= args.warmup:
-                times.append(t); insts += n_i
+        # every step: P = nproc oracle processes (a persistent pool) each simulate whole random
+        # sub-traces of the workload for ~per_step seconds; step time = wall clock of the step
+        import multiprocessing as mp
+        hi = host_info()
+        P = hi["nproc"]
+        per_step = float(os.environ.get("PSIM_REF_STEP_S", "3.0"))
+        times, insts, subs = [], 0, 0
+        with mp.get_context("spawn").Pool(P) as pool:
+            for it in range(args.warmup + args.steps):
+                t0 = time.perf_counter()
+                res = pool.map(_oracle_worker, [(args.config, per_step, 100000 * it + i) for i in range(P)])
+                dt = time.perf_counter() - t0
+                if it >= args.warmup:
+                    times.append(dt); insts += sum(r[0] for r in res); subs += sum(r[2] for r in res)
         tot = sum(times)
         val = insts / tot / 1e6
         line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "MIPS", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic", "config": config,
-                "cpu_baseline": {"value": val, "unit": "MIPS", "cores": 1, "kind": "oracle",
-                                 "sample": f"{insts} instructions of whole random sub-traces of {args.config} per "
-                                           f"{args.steps} steps, single-threaded plain-C oracle"},
+                "cpu_baseline": {"value": val, "unit": "MIPS", "cores": P, "kind": "oracle",
+                                 "sample": f"per step: {P} processes x ~{per_step:.0f} s of whole random sub-traces "
+                                           f"of {args.config} ({insts} counted instructions, {subs} sub-traces over "
+                                           f"{args.steps} timed steps), plain-C oracle "
+                                           + ("bf16-operand" if cfg["precision"] == "bf16" else "fp64") + " mode",
+                                 "host": hi},
                 "e2e": {"value": val, "unit": "MIPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
         return
@@ -359,10 +448,19 @@ def main():
         n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W)
         gcyc = sim.corrections()[1] if args.correction else sim.subtrace_cycles()   # first-pass cycles
         errs = [abs(int(gcyc[j]) - c) / max(c, 1) for j, c in per.items()]
-        line["cpu_baseline"] = {"value": n_i / t / 1e6, "unit": "MIPS", "cores": 1, "kind": "oracle",
-                                "sample": f"{len(per)} whole sub-traces ({n_i} counted instructions, W={W} warm-up "
-                                          f"each) of {args.config}, plain-C oracle "
-                                          f"{'bf16-operand' if cfg['precision'] == 'bf16' else 'fp64'} mode, 1 thread"}
+        n_all, wall_all, P_all, sub_all, rate_all = oracle_all_cores(args.config, args.cpu_budget_all)
+        line["cpu_baseline"] = {"value": rate_all / 1e6, "unit": "MIPS", "cores": P_all, "kind": "oracle",
+                                "sample": f"all host cores: {P_all} oracle processes x ~{args.cpu_budget_all:.0f} s, "
+                                          f"{sub_all} whole random sub-traces ({n_all} counted instructions, W={W} "
+                                          f"warm-up each) of {args.config}; value = sum of per-process rates "
+                                          f"(wall {wall_all:.1f} s incl. start-up)",
+                                "host": host_info(),
+                                "single_thread": {"value": n_i / t / 1e6, "unit": "MIPS", "cores": 1,
+                                                  "sample": f"{len(per)} whole sub-traces ({n_i} counted "
+                                                            f"instructions) of {args.config}, "
+                                                            f"{t:.1f} s"},
+                                "mode": "plain-C oracle, " + ("bf16-operand" if cfg["precision"] == "bf16" else "fp64")
+                                        + " mode, dense CNN"}
         line["parity_sample"] = {"subtraces": sorted(per), "max_rel_cycle_err": max(errs) if errs else None}
     sim.close()
     if rank == 0:
