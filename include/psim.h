@@ -126,7 +126,7 @@ typedef struct {
     double load_ms;           /* device time spent in trace loading before/while stepping  */
     int64_t local_cycles;     /* sum of this rank's sub-trace cycles                       */
     int32_t trace_mode;       /* 0 device-resident, 1 pinned host (zero-copy loader), 2 pageable */
-    int32_t pad;
+    int32_t comm_ranks;       /* ranks of the NCCL communicator the last simulate reduced over (0: none) */
     double kernel_ms[8];      /* PSIM_PROFILE: summed device time per kernel class          */
     uint64_t kernel_launches[8]; /* launches per kernel class                               */
     uint64_t layer_m[4];      /* GEMM rows per launch of layers 0..3 (M = sub-traces x positions) */
@@ -199,6 +199,17 @@ int psim_force_latencies(psim_ctx* ctx, const uint16_t* lat3, uint64_t n_instr);
 int psim_get_rows(const psim_ctx* ctx, uint64_t first, uint64_t n, uint16_t* out3, int32_t* k,
                   int64_t* clock);
 
+/* Raw CNN outputs of the last simulate for real rows [first, first + n) of
+ * this rank: out3 [n][3] fp32 (fetch, complete, store before rounding)
+ * exactly as the hot path computed them (the fused bf16 C3 kernels, the
+ * layer-wise GEMMs or the fp32 SIMT path -- whichever simulate ran), for the
+ * step that predicted each row.  Requires PSIM_RECORD_ROWS and a CNN run
+ * (a model loaded and either no teacher forcing or PSIM_FORCE_PREDICT);
+ * otherwise STATE.  Rows outside this rank's sub-traces are ARG.  Parity
+ * stage S2 of the hot path: with PSIM_FORCE_PREDICT and the oracle's
+ * latencies forced, the inputs are the oracle's, element by element. */
+int psim_get_outputs(const psim_ctx* ctx, uint64_t first, uint64_t n, float* out3);
+
 /* Cycles of local sub-traces [first, first + n) (index relative to this
  * rank's first sub-trace) into out (int64). */
 int psim_get_subtrace_cycles(const psim_ctx* ctx, uint64_t first, uint64_t n, int64_t* out);
@@ -240,7 +251,11 @@ int psim_get_stats(const psim_ctx* ctx, psim_stats* out);
 
 /* Batched CNN forward on caller inputs (parity stage S2): X host [B][112][50]
  * fp32 (the instruction-major input of PAPER.md:93), Y host [B][3] fp32 raw
- * outputs before rounding.  Runs the same kernels as simulate. */
+ * outputs before rounding.  Runs the layer-wise lowering of the loaded model
+ * (gather-free: the inputs are given): per-layer tcgen05 GEMMs for bf16, SIMT
+ * GEMMs for fp32.  The fused bf16 C3 kernels that simulate runs by default
+ * build their inputs from the queue and cannot take caller inputs; their raw
+ * outputs are read with psim_get_outputs. */
 int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float* Y);
 
 /* Name of kernel class i (0 <= i < PSIM_KC_COUNT), or NULL. */

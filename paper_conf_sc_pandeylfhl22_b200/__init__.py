@@ -54,12 +54,12 @@ class Stats(ctypes.Structure):
                 ("simulated", ctypes.c_uint64), ("counted", ctypes.c_uint64), ("subtraces", ctypes.c_uint64),
                 ("h2d_bytes", ctypes.c_uint64), ("gpu_launches", ctypes.c_uint64), ("sim_ms", ctypes.c_double),
                 ("load_ms", ctypes.c_double), ("local_cycles", ctypes.c_int64), ("trace_mode", ctypes.c_int32),
-                ("pad", ctypes.c_int32), ("kernel_ms", ctypes.c_double * 8), ("kernel_launches", ctypes.c_uint64 * 8),
+                ("comm_ranks", ctypes.c_int32), ("kernel_ms", ctypes.c_double * 8), ("kernel_launches", ctypes.c_uint64 * 8),
                 ("layer_m", ctypes.c_uint64 * 4), ("layer_n", ctypes.c_uint32 * 4), ("layer_k", ctypes.c_uint32 * 4),
                 ("corrected", ctypes.c_uint64), ("corr_steps", ctypes.c_uint64)]
 
     def as_dict(self):
-        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "pad"}
+        d = {f: getattr(self, f) for f, _ in self._fields_}
         for f in ("k_hist", "kernel_ms", "kernel_launches", "layer_m", "layer_n", "layer_k"):
             d[f] = list(d[f])
         d["kernel_names"] = [lib().psim_kernel_class_name(i).decode() for i in range(8)]
@@ -70,7 +70,7 @@ EXPORTS = ["psim_create", "psim_destroy", "psim_load_trace", "psim_partition", "
            "psim_simulate", "psim_total_cycles", "psim_last_error", "psim_force_latencies", "psim_get_rows",
            "psim_get_subtrace_cycles", "psim_rank_range", "psim_get_stats", "psim_cnn_forward", "psim_version",
            "psim_partition_range", "psim_kernel_class_name", "psim_nccl_unique_id", "psim_get_corrections",
-           "psim_get_corrected_rows", "psim_get_interval_metrics"]
+           "psim_get_corrected_rows", "psim_get_interval_metrics", "psim_get_outputs"]
 
 _lib = None
 
@@ -96,6 +96,7 @@ def lib():
         L.psim_last_error.restype = c.c_char_p
         L.psim_force_latencies.argtypes = [P, P, c.c_uint64]
         L.psim_get_rows.argtypes = [P, c.c_uint64, c.c_uint64, P, P, P]
+        L.psim_get_outputs.argtypes = [P, c.c_uint64, c.c_uint64, P]
         L.psim_get_subtrace_cycles.argtypes = [P, c.c_uint64, c.c_uint64, P]
         L.psim_get_corrections.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
         L.psim_get_corrected_rows.argtypes = [P, c.c_uint64, c.c_uint64, P, P]
@@ -256,6 +257,12 @@ class Simulator:
         clk = np.zeros(n, np.int64)
         self._check(lib().psim_get_rows(self._h, first, n, _ptr(lat), _ptr(k), _ptr(clk)))
         return lat, k, clk
+
+    def get_outputs(self, first: int, n: int) -> np.ndarray:
+        """Raw fp32 CNN outputs [n][3] the hot path computed for real rows [first, first+n)."""
+        y = np.zeros((max(n, 1), 3), np.float32)
+        self._check(lib().psim_get_outputs(self._h, first, n, _ptr(y)))
+        return y[:n]
 
     def subtrace_cycles(self, first: int = 0, n: int | None = None) -> np.ndarray:
         rr = self.rank_range()

@@ -113,6 +113,8 @@ struct UpdateArgs {
   uint16_t* rec_lat;         // [rows][3] or nullptr (PSIM_RECORD_ROWS)
   int32_t* rec_k;            // [rows] or nullptr
   int64_t* rec_clock;        // [rows] or nullptr
+  float* rec_y = nullptr;    // [rows][3] raw fp32 CNN outputs y of the step that predicted row r
+                             // (PSIM_RECORD_ROWS with a CNN, parity stage S2 of the hot path)
   // post-error correction (R19), entry-major [t][n]:
   uint8_t* k1_rec = nullptr;   // first pass: context count at real row s_b + t, t < limit
   uint32_t* c1_rec = nullptr;  // first pass: Clock - bnd after real row s_b + t

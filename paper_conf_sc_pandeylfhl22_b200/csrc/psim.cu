@@ -161,6 +161,9 @@ struct psim_ctx {
   uint16_t* rec_lat = nullptr;
   int32_t* rec_k = nullptr;
   int64_t* rec_clock = nullptr;
+  float* rec_y = nullptr;       // [rows][3] raw CNN outputs (PSIM_RECORD_ROWS with a CNN)
+  size_t rec_y_cap = 0;
+  bool rec_y_valid = false;
   size_t rec_cap = 0;
   Pec pec;                 // post-error correction (opts.correction_limit > 0)
   bool pec_done = false;
@@ -224,7 +227,9 @@ int psim_create(const psim_opts* opts, psim_ctx** out) {
     ctx->own_stream = true;
   }
   for (auto& e : ctx->ev) cudaEventCreate(&e);
-  if (opts->world_size > 1 && opts->nccl_id) {
+  // a communicator whenever an id is given (also world_size 1: the NCCL leg then runs
+  // as it does on G ranks and must leave the totals unchanged -- tested)
+  if (opts->nccl_id) {
     if (!load_nccl()) { psim_destroy(ctx); return PSIM_ERR_NCCL; }
     ncclUniqueId id;
     memcpy(&id, opts->nccl_id, sizeof id);
@@ -262,6 +267,7 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->rec_lat);
   dfree(ctx->rec_k);
   dfree(ctx->rec_clock);
+  dfree(ctx->rec_y);
   dfree(ctx->fused.T);
   dfree(ctx->fused.w1p);
   dfree(ctx->fused.trace16);
@@ -722,6 +728,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   pf.reset((ctx->opts.flags & PSIM_PROFILE) != 0, st);
   stats.subtraces = n;
   stats.trace_mode = ctx->trace_mode;
+  stats.comm_ranks = ctx->comm ? (int32_t)ctx->opts.world_size : 0;
 
   int rc = ensure_state(ctx);
   if (rc) return rc;
@@ -752,6 +759,13 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     CK(cudaMalloc(&ctx->rec_clock, rows * 8 + 8));
     ctx->rec_cap = rows;
   }
+  if (rec && predict && ctx->rec_y_cap < (size_t)rows) {
+    dfree(ctx->rec_y);
+    ctx->rec_y = nullptr;
+    CK(cudaMalloc(&ctx->rec_y, rows * 12 + 16));
+    ctx->rec_y_cap = rows;
+  }
+  ctx->rec_y_valid = rec && predict;
   if (forced) {
     if (ctx->d_forced_cap < (size_t)rows) {
       dfree(ctx->d_forced);
@@ -824,6 +838,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   UpdateArgs ua{ctx->st, ctx->row_lo, 0, ctx->cap, predict ? ctx->buf.y : nullptr,
                 forced ? ctx->d_forced : nullptr, rec ? ctx->rec_lat : nullptr, rec ? ctx->rec_k : nullptr,
                 rec ? ctx->rec_clock : nullptr};
+  ua.rec_y = (rec && predict) ? ctx->rec_y : nullptr;
   if (pec) { ua.k1_rec = ctx->pec.k1; ua.c1_rec = ctx->pec.c1; ua.limit = ctx->pec.limit; }
   if (metrics) {
     // per-row metric codes: from the device-visible uint8 rows, or written by the
@@ -1013,6 +1028,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     u2.rec_lat = rec ? p.rec_lat : nullptr;
     u2.rec_k = rec ? p.rec_k : nullptr;
     u2.rec_clock = nullptr;
+    u2.rec_y = nullptr;   // recorded outputs stay the first pass's
     if (rec) {
       CK(cudaMemsetAsync(p.rec_lat, 0, rows * 6, st));
       CK(cudaMemsetAsync(p.rec_k, 0xFF, rows * 4, st));
@@ -1165,6 +1181,19 @@ extern "C" int psim_get_rows(const psim_ctx* cctx, uint64_t first, uint64_t n, u
   if (out3) CK(cudaMemcpy(out3, ctx->rec_lat + 3 * off, n * 6, cudaMemcpyDeviceToHost));
   if (k) CK(cudaMemcpy(k, ctx->rec_k + off, n * 4, cudaMemcpyDeviceToHost));
   if (clock) CK(cudaMemcpy(clock, ctx->rec_clock + off, n * 8, cudaMemcpyDeviceToHost));
+  return PSIM_OK;
+}
+
+extern "C" int psim_get_outputs(const psim_ctx* cctx, uint64_t first, uint64_t n, float* out3) {
+  psim_ctx* ctx = const_cast<psim_ctx*>(cctx);
+  if (!ctx || !out3) return PSIM_ERR_ARG;
+  if (!ctx->done) FAIL(PSIM_ERR_STATE, "no simulate yet");
+  if (!ctx->rec_y_valid) FAIL(PSIM_ERR_STATE, "no recorded CNN outputs (needs PSIM_RECORD_ROWS and a CNN run)");
+  const int64_t s_first = ctx->h_s.empty() ? 0 : ctx->h_s.front();
+  if ((int64_t)first < s_first || (int64_t)(first + n) > ctx->row_hi) FAIL(PSIM_ERR_ARG, "rows outside this rank");
+  const int64_t off = (int64_t)first - ctx->row_lo;
+  CK(cudaSetDevice(ctx->opts.device));
+  CK(cudaMemcpy(out3, ctx->rec_y + 3 * off, n * 12, cudaMemcpyDeviceToHost));
   return PSIM_OK;
 }
 

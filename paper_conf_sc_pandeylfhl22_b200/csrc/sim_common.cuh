@@ -160,6 +160,7 @@ __device__ __forceinline__ int update_subtrace(const UpdateArgs& a, uint64_t b, 
       if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
       if (a.rec_k) a.rec_k[r] = k;
       if (a.rec_clock) a.rec_clock[r] = clock;
+      if (a.rec_y) { a.rec_y[3 * r] = y0; a.rec_y[3 * r + 1] = y1; a.rec_y[3 * r + 2] = y2; }
     }
   }
   return base;
@@ -286,6 +287,7 @@ done:
     if (a.rec_lat) { a.rec_lat[3 * r] = (uint16_t)pf; a.rec_lat[3 * r + 1] = (uint16_t)pc; a.rec_lat[3 * r + 2] = (uint16_t)ps; }
     if (a.rec_k) a.rec_k[r] = k;
     if (a.rec_clock) a.rec_clock[r] = clock;
+    if (a.rec_y) { a.rec_y[3 * r] = y0; a.rec_y[3 * r + 1] = y1; a.rec_y[3 * r + 2] = y2; }
   }
   return w;
 }

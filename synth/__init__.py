@@ -118,6 +118,23 @@ FEATURE_SCALE = np.array(
 assert FEATURE_SCALE.size == 50
 
 
+# Completion-latency floor of the synthetic head (R21): the completion row of
+# fc2 is drawn non-negative and its bias is COMPLETE_BIAS > 0.5, so y_c = COMPLETE_BIAS +
+# a sum of non-negative terms (ReLU outputs x non-negative weights) and every rounded
+# completion latency is >= 1.  Every pushed entry then lives at least one cycle, so a
+# Clock that does not advance grows the queue by one entry per instruction and the
+# ROB-full stall (R5) advances it within Context_length instructions: the random-weight
+# model has no frozen-Clock fixed point (round 1 found one at row ~3.3M of the config-4
+# trace: f = c = s = 0 with an unchanging context for millions of rows).
+# Applied to the models of the long-running configs (C3: configs 2-4, RB7: config 5).  M2
+# (config 1: 10k rows, one sub-trace) keeps a signed completion row: with the floor its
+# small network has a positive feedback through the time features (completions run away
+# to the 4095 clamp within ~1k rows), and config 1 is short.
+FLOOR_OUTPUT = 1
+COMPLETE_BIAS = 0.75
+FLOOR_ARCHS = ("C3", "RB7")
+
+
 def calibration(arch: str):
     path = os.path.join(_HERE, "calibration.json")
     if os.path.exists(path):
@@ -145,8 +162,12 @@ def weights(arch: str = "C3", seed: int = WEIGHT_SEED, *, gain=None, bias=None) 
         if li == 0:
             w = w / FEATURE_SCALE[None, :, None]
         if li == len(shapes) - 1:                            # calibrated head
+            if arch in FLOOR_ARCHS:
+                w[FLOOR_OUTPUT] = np.abs(w[FLOOR_OUTPUT])    # completion row non-negative (R21)
             w = w * gain[:, None] / np.sqrt(3.0)
             b = bias.copy()
+            if arch in FLOOR_ARCHS:
+                b[FLOOR_OUTPUT] = COMPLETE_BIAS
         parts += [w.ravel(), b.ravel()]
     out = np.concatenate(parts).astype(np.float32)
     assert out.size == nparams(arch)

@@ -23,9 +23,15 @@ pytestmark = pytest.mark.gpu
 
 
 def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, forced=None,
-            record=True, rank=0, world=1, first_row=0, n_instr=None, device_trace=False, layerwise=False):
-    with P.Simulator(precision=precision, queue_cap=cap, record_rows=record, rank=rank,
-                     world_size=world, layerwise=layerwise) as sim:
+            record=True, rank=0, world=1, first_row=0, n_instr=None, device_trace=False, layerwise=False,
+            variant="warp"):
+    """variant (teacher-forced runs): "warp" = the standalone warp-per-sub-trace update
+    kernel; "fused" = the thread-per-sub-trace update inside fc1_head_kernel (the hot
+    path), reached by running the fused C3 CNN with PSIM_FORCE_PREDICT while the queue
+    follows the forced latencies."""
+    fused_forced = forced is not None and variant == "fused"
+    with P.Simulator(precision="bf16" if fused_forced else precision, queue_cap=cap, record_rows=record, rank=rank,
+                     world_size=world, layerwise=layerwise, force_predict=fused_forced) as sim:
         if device_trace:
             t = torch.from_numpy(np.ascontiguousarray(trace)).cuda()
             sim.load_trace(t, n_instr=n_instr, first_row=first_row)
@@ -34,6 +40,8 @@ def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, 
         sim.partition(N, W)
         if forced is not None:
             sim.force_latencies(forced)
+            if fused_forced:
+                sim.load_model("C3", synth.weights("C3"))
         else:
             sim.load_model(arch, weights)
         sim.simulate()
@@ -48,28 +56,36 @@ def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, 
 
 
 # ------------------------------------------------------------------ S1
-def test_s1_hand_trace_partitions():
+VARIANTS = ["warp", "fused"]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_s1_hand_trace_partitions(variant):
     from test_oracle_queue import distinct_trace, parse_golden
     rows, parts = parse_golden()
     lat = np.array([r["lat"] for r in rows], np.uint16)
     tr = distinct_trace(20)
     for W, cyc, total in parts:
-        g = gpu_run(tr, 4, W, cap=4, forced=lat)
+        g = gpu_run(tr, 4, W, cap=4, forced=lat, variant=variant)
         assert g["cycles"].tolist() == cyc and g["total"] == total
-    g = gpu_run(tr, 1, 0, cap=4, forced=lat)
+    g = gpu_run(tr, 1, 0, cap=4, forced=lat, variant=variant)
     assert g["total"] == 69
     assert g["clock"].tolist() == [r["clock_out"] for r in rows]
     assert g["k"].tolist() == [len(r["ctx"]) for r in rows]
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("L,N,W,cap,big", [
     (6000, 1, 0, 110, 0.0), (6000, 37, 50, 8, 0.02), (6000, 6000, 3, 110, 0.0),
-    (5000, 333, 1000, 1, 0.0), (7919, 64, 110, 110, 0.05), (4096, 128, 0, 17, 0.01)])
-def test_s1_teacher_forced_bit_exact(L, N, W, cap, big):
+    (5000, 333, 1000, 1, 0.0), (7919, 64, 110, 110, 0.05), (4096, 128, 0, 17, 0.01),
+    (60_000, 301, 40, 110, 0.3)])
+def test_s1_teacher_forced_bit_exact(L, N, W, cap, big, variant):
+    """The last case saturates the queues (30% of completions up to 4095 cycles): ROB-full
+    stalls, k = 110 and all 14 conv3 positions on the fused path, ragged tiles (N = 301)."""
     tr = synth.trace(L, 4242 + N)
     lat = synth.teacher_latencies(L, 99 + N, c_mean=30.0 if cap > 20 else 5.0, big=big)
     ref = oracle.simulate(tr, N, W, forced_lat=lat, cap=cap)
-    g = gpu_run(tr, N, W, cap=cap, forced=lat)
+    g = gpu_run(tr, N, W, cap=cap, forced=lat, variant=variant)
     assert np.array_equal(g["k"], ref["k"])
     assert np.array_equal(g["clock"], ref["clock"])
     assert np.array_equal(g["cycles"], ref["cycles"])
@@ -77,16 +93,17 @@ def test_s1_teacher_forced_bit_exact(L, N, W, cap, big):
     assert g["stats"]["stalls"] == ref["stalls"]
 
 
-def test_s1_clock_beyond_32_bits():
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_s1_clock_beyond_32_bits(variant):
     # fetch latencies at the clamp (4095) push the Clock past 2^32: the low-32-bit
-    # age arithmetic must stay exact.
+    # age arithmetic (and the fused update's rmin fast path) must stay exact.
     L = 1_100_000
     tr = np.zeros((L, 48), np.uint8)
     lat = synth.teacher_latencies(L, 5, c_mean=30.0)
     lat[:, 0] = 4095
     ref = oracle.simulate(tr, 1, 0, forced_lat=lat, cap=110)
     assert ref["clock"].max() > 2**32
-    g = gpu_run(tr, 1, 0, forced=lat)
+    g = gpu_run(tr, 1, 0, forced=lat, variant=variant)
     assert np.array_equal(g["clock"], ref["clock"]) and np.array_equal(g["k"], ref["k"])
     assert g["total"] == ref["total"]
 
@@ -193,17 +210,53 @@ def test_s2_cnn_bf16_tensor_cores(arch):
 # So S3 is split: (a) decision agreement -- the GPU's gather + CNN + rounding on
 # the ORACLE's trajectory (teacher-forced queue, PSIM_FORCE_PREDICT) must agree
 # on >= 99.9% of per-instruction (f, c, s); (b) free-running totals within 0.5%.
-def decision_parity(tr, N, arch, w, precision, samples=None, cap=110, layerwise=False):
-    """W = 0 so the per-row forced latencies are exactly each sub-trace's oracle trajectory."""
+# S2 tolerances of the raw outputs y, max|dy| / max(|y|, 1) per row, GPU vs the oracle of the
+# same precision.  fp32 path vs the fp64 oracle: 1e-3 (north_star).  bf16 path vs the
+# bf16-operand oracle: same rounding points, different summation order (fp32 in the tensor
+# core vs exact), so an intermediate activation within fp32 noise of a bf16 rounding
+# boundary can round one bf16 ulp (2^-8) the other way (R15) and carry that into y: the
+# worst row is bounded at 5e-3 and the TYPICAL row must agree to fp32 precision (median
+# <= 1e-5); against the fp64 oracle the north_star bound 2e-2 holds for every row.
+Y_TOL = {"fp32": 1e-3, "bf16": 5e-3}
+Y_MEDIAN = 1e-5
+
+
+def _legit_flip(yg, yr, lg, lr, y_tol):
+    """R15: a disagreeing rounded latency is legitimate iff the GPU's and the oracle's raw
+    outputs agree within S2's tolerance -- they then straddle the rounding boundary
+    between the two integers."""
+    for o in range(3):
+        if lg[o] == lr[o]:
+            continue
+        if abs(float(yg[o]) - float(yr[o])) > y_tol * max(abs(float(yr[o])), 1.0):
+            return False
+        lo, hi = sorted((int(lg[o]), int(lr[o])))
+        if hi - lo != 1:
+            return False
+        b = lo + 0.5                                   # the boundary both sides are next to
+        if not (min(yg[o], yr[o]) - 1e-6 * max(abs(b), 1.0) <= b <= max(yg[o], yr[o]) + 1e-6 * max(abs(b), 1.0)):
+            return False
+    return True
+
+
+def decision_parity(tr, N, arch, w, precision, samples=None, cap=110, layerwise=False, y_tol=None):
+    """W = 0 so the per-row forced latencies are exactly each sub-trace's oracle trajectory.
+    The GPU's gather + CNN + rounding run on that trajectory (PSIM_FORCE_PREDICT); its raw
+    outputs y are recorded by the hot path itself.  Returns a dict: agreement of the rounded
+    (f, c, s), the S2 error of y on every compared row (element-wise, vs the oracle of the
+    same precision), and every disagreement classified (legitimate = R15 boundary case)."""
     L = tr.shape[0]
+    y_tol = Y_TOL[precision] if y_tol is None else y_tol
     mode = oracle.BF16 if precision == "bf16" else oracle.FP64
     forced = synth.teacher_latencies(L, 17)
+    ref_y = np.zeros((L, 3), np.float32)
     rows = []
     js = range(N) if samples is None else samples
     for j in js:
         ref = oracle.simulate(tr, N, 0, arch=arch, weights=w, mode=mode, j0=j, nj=1, cap=cap)
         s, e = j * L // N, (j + 1) * L // N
         forced[s:e] = ref["lat"][s:e]
+        ref_y[s:e] = ref["y"][s:e]
         rows.append((s, e))
     with P.Simulator(precision=precision, record_rows=True, force_predict=True, queue_cap=cap,
                      layerwise=layerwise) as sim:
@@ -212,26 +265,54 @@ def decision_parity(tr, N, arch, w, precision, samples=None, cap=110, layerwise=
         sim.load_model(arch, w)
         sim.force_latencies(forced)
         sim.simulate()
-        agree, n = 0, 0
+        agree, n, legit, bad, yrow = 0, 0, 0, [], []
         for s, e in rows:
             lat, _, _ = sim.get_rows(s, e - s)
-            agree += int(np.sum(np.all(lat == forced[s:e], axis=1)))
+            yg = sim.get_outputs(s, e - s)
+            yr = ref_y[s:e]
+            yrow.append(np.max(np.abs(yg - yr), axis=1) / np.maximum(np.max(np.abs(yr), axis=1), 1.0))
+            eq = np.all(lat == forced[s:e], axis=1)
+            agree += int(np.sum(eq))
             n += e - s
-    return agree / n
+            for r in np.nonzero(~eq)[0]:
+                if _legit_flip(yg[r], yr[r], lat[r], forced[s + r], y_tol):
+                    legit += 1
+                else:
+                    bad.append((s + r, lat[r].tolist(), forced[s + r].tolist(), yg[r].tolist(), yr[r].tolist()))
+    yrow = np.concatenate(yrow)
+    return dict(agree=agree / n, legit=legit, bad=bad, n=n, y_err=float(yrow.max()), y_med=float(np.median(yrow)),
+                y_over_1e4=float(np.mean(yrow > 1e-4)), y_tol=y_tol)
+
+
+def check_decisions(d, min_agree=0.999):
+    print(f"decisions: agree {d['agree']:.5f} legit flips {d['legit']} of {d['n']}, y err max {d['y_err']:.2e} "
+          f"median {d['y_med']:.2e}, rows > 1e-4: {d['y_over_1e4']:.4f}")
+    assert not d["bad"], f"disagreements not at a rounding boundary: {d['bad'][:5]}"
+    assert d["y_err"] <= d["y_tol"] and d["y_med"] <= Y_MEDIAN, d
+    assert d["agree"] >= min_agree, d
 
 
 def free_running(tr, N, W, arch, w, precision, samples=None, layerwise=False):
+    """Free-running GPU vs oracle on the same N, W.  Returns (aggregate relative cycle
+    error over the sampled sub-traces, free-running per-instruction agreement, gpu run,
+    per-sub-trace details).  A sub-trace whose every rounded latency agrees with the
+    oracle must have bit-identical cycles (same trajectory)."""
     L = tr.shape[0]
     mode = oracle.BF16 if precision == "bf16" else oracle.FP64
     g = gpu_run(tr, N, W, arch=arch, weights=w, precision=precision, layerwise=layerwise)
     js = list(range(N)) if samples is None else list(samples)
-    ref_c, gpu_c, agree, n = 0, 0, 0, 0
+    ref_c, gpu_c, agree, n, per = 0, 0, 0, 0, []
     for j in js:
         ref = oracle.simulate(tr, N, W, arch=arch, weights=w, mode=mode, j0=j, nj=1)
         s, e = j * L // N, (j + 1) * L // N
-        ref_c += int(ref["cycles"][0]); gpu_c += int(g["cycles"][j])
-        agree += int(np.sum(np.all(g["lat"][s:e] == ref["lat"][s:e], axis=1))); n += e - s
-    return abs(gpu_c - ref_c) / ref_c, agree / n, g
+        rc, gc = int(ref["cycles"][0]), int(g["cycles"][j])
+        ref_c += rc; gpu_c += gc
+        a = int(np.sum(np.all(g["lat"][s:e] == ref["lat"][s:e], axis=1)))
+        agree += a; n += e - s
+        if a == e - s:
+            assert gc == rc, (j, gc, rc)
+        per.append((j, a / (e - s), abs(gc - rc) / max(rc, 1)))
+    return abs(gpu_c - ref_c) / ref_c, agree / n, g, per
 
 
 def test_s3_config1_m2_fp32():
@@ -240,8 +321,9 @@ def test_s3_config1_m2_fp32():
     L = 10_000
     tr = synth.trace(L, synth.TRACE_SEED_BASE + 0)
     w = synth.weights("M2")
-    assert decision_parity(tr, 1, "M2", w, "fp32") >= 0.999
-    rel, agree, _ = free_running(tr, 1, 0, "M2", w, "fp32")
+    check_decisions(decision_parity(tr, 1, "M2", w, "fp32"))
+    rel, agree, _, per = free_running(tr, 1, 0, "M2", w, "fp32")
+    print(f"config1: free-running per-instruction agreement {agree:.5f}, total error {rel:.2e}")
     assert rel <= 0.005
 
 
@@ -252,51 +334,68 @@ def test_s3_c3_small(precision, layerwise):
     L, N = 3000, 6
     tr = synth.trace(L, 2024)
     w = synth.weights("C3")
-    assert decision_parity(tr, N, "C3", w, precision, layerwise=layerwise) >= 0.999
-    rel, agree, _ = free_running(tr, N, 64, "C3", w, precision, layerwise=layerwise)
-    assert rel <= 0.005, (rel, agree)
+    check_decisions(decision_parity(tr, N, "C3", w, precision, layerwise=layerwise))
+    rel, agree, _, per = free_running(tr, N, 64, "C3", w, precision, layerwise=layerwise)
+    print(f"C3 small {precision} layerwise={layerwise}: free-running agreement {agree:.5f}, total error {rel:.2e}")
+    assert rel <= 0.005, (rel, agree, per)
 
 
-def test_s3_fused_full_queue_and_ragged_tiles():
-    """Fused path: contexts filled to the 110-entry cap (all 14 conv3 positions
-    computed, P = 14) by long completion latencies, ragged sub-trace counts
-    (N = 300: tiles of 128 + a partial tile) and finished sub-traces (ragged lengths)."""
-    L, N = 45_017, 300                      # ~150 instructions per sub-trace, ragged
-    tr = synth.trace(L, 99)
+def test_s2_fused_hot_path_outputs():
+    """S2 on the HOT PATH: the raw fp32 outputs y of the fused conv_stack + fc1_head
+    kernels (recorded by fc1_head as it computes them, psim_get_outputs), element by
+    element against the oracle's CNN on the same inputs: <= 1e-3 vs the bf16-operand
+    oracle and <= 2e-2 vs the fp64 oracle (north_star).  The queues follow forced
+    latencies (PSIM_FORCE_PREDICT), so the inputs are the oracle's.  Covers k = 0 (the
+    first row of every sub-trace), contexts filled to the 110-entry cap (P = 14, ROB-full
+    stalls) in every third sub-trace, ragged sub-trace lengths and a ragged last tile
+    (N = 20003), and ~7 conv tiles per CTA per step (every pipeline ring wraps)."""
+    N, per = 20_003, 150
+    L = N * per + 17
+    tr = synth.trace(L, 6061)
     w = synth.weights("C3")
-    forced = synth.teacher_latencies(L, 23, c_mean=400.0)        # queues saturate: k -> 110, stalls
-    mode = oracle.BF16
-    refs = {}
-    for j in (0, 7, 128, 255, 299):
-        ref = oracle.simulate(tr, N, 0, forced_lat=forced, j0=j, nj=1, cap=110)
-        refs[j] = ref
-    # decision agreement of the CNN on those saturated trajectories
+    forced = synth.teacher_latencies(L, 29, c_mean=30.0)
+    sat = synth.teacher_latencies(L, 31, c_mean=400.0, big=0.3)
+    bounds = [(j * L // N, (j + 1) * L // N) for j in range(N)]
+    for j in range(0, N, 3):                       # saturating sub-traces
+        s_, e_ = bounds[j]
+        forced[s_:e_] = sat[s_:e_]
+    samples = [0, 3, 127, 128, 300, 9999, 20001, 20002]
     with P.Simulator(precision="bf16", record_rows=True, force_predict=True) as sim:
         sim.load_trace(tr); sim.partition(N, 0); sim.load_model("C3", w); sim.force_latencies(forced)
         sim.simulate()
         st = sim.stats()
         assert max(i for i, c in enumerate(st["k_hist"]) if c) == 110
-        agree, legit, n, bad = 0, 0, 0, []
-        for j in refs:
-            s, e = j * L // N, (j + 1) * L // N
-            lat, k, clk = sim.get_rows(s, e - s)
-            assert np.array_equal(k, refs[j]["k"][s:e]) and np.array_equal(clk, refs[j]["clock"][s:e])
+        assert st["layer_m"][0] / 128 / 148 > 5            # mean conv tiles per CTA per step
+        e16, e64 = [], 0.0
+        ks = set()
+        agree = n = 0
+        for j in samples:
+            s_, e_ = bounds[j]
+            lat, k, _ = sim.get_rows(s_, e_ - s_)
+            yg = sim.get_outputs(s_, e_ - s_)
             q = oracle.Queue(110)
-            for i in range(s, e):            # the oracle's own CNN decision on the same state
+            for i in range(s_, e_):
                 X, kk = q.build_input(tr, i)
-                y = oracle.cnn_forward("C3", w, X, mode=mode)
-                ref = tuple(oracle.round_latency(v) for v in y)
-                got = tuple(int(v) for v in lat[i - s])
+                assert kk == k[i - s_]
+                ks.add(kk)
+                y16 = oracle.cnn_forward("C3", w, X, mode=oracle.BF16)
+                y64 = oracle.cnn_forward("C3", w, X)
+                g = yg[i - s_]
+                e16.append(float(np.max(np.abs(g - y16)) / max(float(np.max(np.abs(y16))), 1.0)))
+                e64 = max(e64, float(np.max(np.abs(g - y64)) / max(float(np.max(np.abs(y64))), 1.0)))
+                ref = [oracle.round_latency(v) for v in y16]
                 n += 1
-                if ref == got:
+                if ref == [int(v) for v in lat[i - s_]]:
                     agree += 1
-                elif all(r == g or abs(abs(v - np.floor(v)) - 0.5) <= 1e-3 * max(abs(v), 1.0)
-                         for r, g, v in zip(ref, got, y)):
-                    legit += 1                   # R15: within S2's tolerance of a .5 boundary
                 else:
-                    bad.append((i, kk, ref, got, y))
+                    assert _legit_flip(g, np.asarray(y16, np.float32), lat[i - s_], ref, Y_TOL["bf16"]), (i, g, y16)
                 q.update(i, *(int(v) for v in forced[i]))
-        assert not bad and (agree + legit) / n >= 0.999 and agree / n >= 0.99, (agree, legit, n, bad[:5])
+    assert 0 in ks and 110 in ks
+    e16 = np.array(e16)
+    print(f"S2 fused: err vs bf16 oracle max {e16.max():.2e} median {np.median(e16):.2e} (rows > 1e-4: "
+          f"{np.mean(e16 > 1e-4):.4f}), vs fp64 oracle max {e64:.2e}, decisions {agree}/{n}")
+    assert e16.max() <= Y_TOL["bf16"] and np.median(e16) <= Y_MEDIAN and e64 <= 2e-2
+    assert agree / n >= 0.999
 
 
 def test_s3_config2_full_size_sampled():
@@ -306,9 +405,10 @@ def test_s3_config2_full_size_sampled():
     L, N = 1_000_000, 1024
     tr = synth.trace(L, synth.TRACE_SEED_BASE + 1)
     w = synth.weights("C3")
-    assert decision_parity(tr, N, "C3", w, "bf16", samples=[0, 333, 517, 1023]) >= 0.999
-    rel, agree, g = free_running(tr, N, 1000, "C3", w, "bf16", samples=[0, 201, 517, 640, 700, 967, 1023])
-    assert rel <= 0.005, (rel, agree)
+    check_decisions(decision_parity(tr, N, "C3", w, "bf16", samples=[0, 333, 517, 1023]))
+    rel, agree, g, per = free_running(tr, N, 1000, "C3", w, "bf16", samples=[0, 201, 517, 640, 700, 967, 1023])
+    print(f"config2: free-running agreement {agree:.5f}, total error {rel:.2e}, per sub-trace {per}")
+    assert rel <= 0.005, (rel, agree, per)
     assert g["stats"]["counted"] == L
 
 
@@ -319,9 +419,10 @@ def test_s3_config3_full_size_sampled():
     L, N = 100_000_000, 65536
     tr = synth.trace(L, synth.TRACE_SEED_BASE + 2)
     w = synth.weights("C3")
-    assert decision_parity(tr, N, "C3", w, "bf16", samples=[0, 40000, 65535]) >= 0.999
-    rel, agree, g = free_running(tr, N, 110, "C3", w, "bf16", samples=[0, 1, 9999, 32768, 40000, 65535])
-    assert rel <= 0.005, (rel, agree)
+    check_decisions(decision_parity(tr, N, "C3", w, "bf16", samples=[0, 40000, 65535]))
+    rel, agree, g, per = free_running(tr, N, 110, "C3", w, "bf16", samples=[0, 1, 9999, 32768, 40000, 65535])
+    print(f"config3: free-running agreement {agree:.5f}, total error {rel:.2e}, per sub-trace {per}")
+    assert rel <= 0.005, (rel, agree, per)
 
 
 @pytest.mark.parametrize("chunk", [0, 7])

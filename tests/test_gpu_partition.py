@@ -33,3 +33,30 @@ def test_partition_error_trends():
     for N in (256, 4096, 16384):
         assert abs(err[(N, 128)]) < 0.03, err
         assert abs(err[(N, 128)]) < abs(err[(N, 0)]) or abs(err[(N, 0)]) < 0.01, err
+
+
+def test_nccl_one_rank_communicator_leaves_results_unchanged():
+    """The NCCL leg (one reduction at the end) executed for real: a 1-rank
+    communicator built from psim_nccl_unique_id (the same call sequence a G-rank job
+    uses) must give the same total and the same interval metrics as a run without a
+    communicator (the fake-backend equivalent on one GPU).  NCCL cannot
+    place two ranks on one device, so G > 1 is covered by the gloo host test and the
+    emulated rank slices."""
+    import numpy as np
+    import synth
+    L, N, W, I = 30_000, 96, 64, 500
+    tr = synth.trace(L, 8181)
+    w = synth.weights("C3")
+    res = []
+    for nid in (None, P.nccl_unique_id()):
+        with P.Simulator(precision="bf16", interval=I, nccl_id=nid) as sim:
+            sim.load_trace(tr)
+            sim.partition(N, W)
+            sim.load_model("C3", w)
+            sim.simulate()
+            res.append((sim.total_cycles(), sim.subtrace_cycles(), sim.interval_metrics(), sim.stats()["comm_ranks"]))
+    (t0, c0, m0, r0), (t1, c1, m1, r1) = res
+    assert r0 == 0 and r1 == 1
+    assert t0 == t1 == int(c0.sum()) and np.array_equal(c0, c1)
+    for k in ("cycles", "retired", "retired_st", "mem_bytes"):
+        assert np.array_equal(m0[k], m1[k])

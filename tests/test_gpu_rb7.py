@@ -19,7 +19,7 @@ import torch
 import oracle
 import paper_conf_sc_pandeylfhl22_b200 as P
 import synth
-from test_gpu_parity import decision_parity, free_running, s2_err, s2_inputs
+from test_gpu_parity import check_decisions, decision_parity, free_running, s2_err, s2_inputs
 
 pytestmark = pytest.mark.gpu
 
@@ -51,48 +51,21 @@ def test_rb7_fp32_unsupported():
         assert e.value.code == P.ERR_UNSUPPORTED
 
 
-def rb7_decisions(tr, N, w, samples, tol=5e-3):
-    """Decision agreement on the oracle's trajectory (W = 0, PSIM_FORCE_PREDICT), as
-    test_gpu_parity.decision_parity, plus the count of LEGITIMATE disagreements: the
-    oracle's output lies within the S2 bound (tol, relative) of a .5 rounding boundary,
-    where a bf16 rounding flip inside the 8-layer network may decide either way (R15)."""
-    L = tr.shape[0]
-    forced = synth.teacher_latencies(L, 17)
-    refs = {}
-    for j in samples:
-        ref = oracle.simulate(tr, N, 0, arch="RB7", weights=w, mode=oracle.BF16, j0=j, nj=1)
-        s, e = j * L // N, (j + 1) * L // N
-        forced[s:e] = ref["lat"][s:e]
-        refs[j] = (s, e, ref["y"][s:e])
-    with P.Simulator(precision="bf16", record_rows=True, force_predict=True) as sim:
-        sim.load_trace(tr)
-        sim.partition(N, 0)
-        sim.load_model("RB7", w)
-        sim.force_latencies(forced)
-        sim.simulate()
-        agree = legit = n = 0
-        bad = []
-        for j, (s, e, y) in refs.items():
-            lat, _, _ = sim.get_rows(s, e - s)
-            for r in range(e - s):
-                n += 1
-                if np.array_equal(lat[r], forced[s + r]):
-                    agree += 1
-                elif all(int(g) == int(f) or abs(abs(v - np.floor(v)) - 0.5) <= tol * max(abs(v), 1.0)
-                         for g, f, v in zip(lat[r], forced[s + r], y[r])):
-                    legit += 1
-                else:
-                    bad.append((s + r, lat[r].tolist(), forced[s + r].tolist(), y[r].tolist()))
-    return agree, legit, n, bad
+def rb7_decisions(tr, N, w, samples):
+    """Decision agreement on the oracle's trajectory (W = 0, PSIM_FORCE_PREDICT) with the
+    hot path's recorded raw outputs compared element by element (test_gpu_parity.
+    decision_parity) at RB7's S2 bound vs the bf16-operand oracle (5e-3, see
+    test_s2_rb7_bf16_tensor_cores); every disagreement must be a rounding-boundary case
+    (R15)."""
+    return decision_parity(tr, N, "RB7", w, "bf16", samples=samples)
 
 
 def test_s3_rb7_small():
     L, N = 1200, 4
     tr = synth.trace(L, 5055)
     w = synth.weights("RB7")
-    agree, legit, n, bad = rb7_decisions(tr, N, w, range(N))
-    assert not bad and (agree + legit) / n >= 0.999 and agree / n >= 0.99, (agree, legit, n, bad[:5])
-    rel, _, _ = free_running(tr, N, 40, "RB7", w, "bf16")
+    check_decisions(rb7_decisions(tr, N, w, range(N)))
+    rel, _, _, _ = free_running(tr, N, 40, "RB7", w, "bf16")
     assert rel <= 0.005, rel
 
 
@@ -103,8 +76,7 @@ def test_s3_rb7_config5_shape():
     L, N = 1_000_000, 512
     tr = synth.trace(L, synth.TRACE_SEED_BASE + 4)
     w = synth.weights("RB7")
-    agree, legit, n, bad = rb7_decisions(tr, N, w, (0, 511))
-    assert not bad and (agree + legit) / n >= 0.999 and agree / n >= 0.99, (agree, legit, n, bad[:5])
+    check_decisions(rb7_decisions(tr, N, w, (0, 511)))
     pinned = torch.from_numpy(tr).pin_memory()
     with P.Simulator(precision="bf16", chunk_steps=256) as sim:
         sim.load_trace(pinned)

@@ -21,7 +21,7 @@ import synth  # noqa: E402
 
 TARGET_MEAN = np.array([1.3, 30.0, 2.0])
 TARGET_STD = np.array([0.7, 10.0, 2.0])
-ITERS = 14
+ITERS = 20
 N_PER_PHASE = {"M2": 150, "C3": 120, "RB7": 60}
 
 
@@ -45,12 +45,22 @@ def main(archs):
             r = oracle.simulate(tr, 8, 0, arch=arch, weights=w)
             y = r["y"].astype(np.float64)
             z = (y - bias) / gain                      # head output at gain 1, bias 0
+            g_prev = gain.copy()
             if it == 0:                                # first: standardise the empty-context outputs
                 gain = TARGET_STD / np.maximum(z.std(0), 1e-9) * 0.05
                 bias = TARGET_MEAN - gain * z.mean(0)
             else:                                      # damped fixed point (feedback through the queue)
                 gain = gain * np.clip(TARGET_STD / np.maximum(y.std(0), 1e-9), 0.5, 2.0) ** 0.5
                 bias = bias + 0.5 * (TARGET_MEAN - y.mean(0))
+            # completion (R21): bias fixed at COMPLETE_BIAS, non-negative row; the gain sets the mean
+            o, b0 = synth.FLOOR_OUTPUT, synth.COMPLETE_BIAS
+            if arch not in synth.FLOOR_ARCHS:
+                o = None
+            zf = None if o is None else = (y[:, o] - b0) / g_prev[o]               # non-negative part at gain 1
+            if o is not None:
+                gain[o] = (TARGET_MEAN[o] - b0) / max(zf.mean(), 1e-9) if it == 0 else \
+                    g_prev[o] * np.clip((TARGET_MEAN[o] - b0) / max(y[:, o].mean() - b0, 1e-9), 0.5, 2.0) ** 0.5
+                bias[o] = b0
             lat = r["lat"].astype(np.float64)
             print(f"{arch} it{it}: y mean {y.mean(0).round(3)} std {y.std(0).round(3)} | "
                   f"lat mean {lat.mean(0).round(3)} | k mean {r['k'].mean():.1f} max {r['k'].max()}"
