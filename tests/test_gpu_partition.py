@@ -60,3 +60,30 @@ def test_nccl_one_rank_communicator_leaves_results_unchanged():
     assert t0 == t1 == int(c0.sum()) and np.array_equal(c0, c1)
     for k in ("cycles", "retired", "retired_st", "mem_bytes"):
         assert np.array_equal(m0[k], m1[k])
+
+
+def test_long_unpartitioned_run_has_no_frozen_clock():
+    """DESIGN.md R21 on the hot path over 1M unpartitioned rows of the config-4 trace (round
+    1's model froze at row ~3.3M): the Clock never stands still for more than
+    Context_length consecutive instructions, every completion latency is >= 1, and the
+    statistics stay SPEC-like over the whole run (CPI, occupancy per 100k-row window)."""
+    import numpy as np
+    import synth
+    L = 1_000_000
+    tr = synth.trace(L, synth.TRACE_SEED_BASE + 3)
+    w = synth.weights("C3")
+    with P.Simulator(precision="bf16", record_rows=True) as sim:
+        sim.load_trace(tr)
+        sim.partition(1, 0)
+        sim.load_model("C3", w)
+        sim.simulate()
+        lat, k, clk = sim.get_rows(0, L)
+    assert lat[:, 1].min() >= 1
+    adv = np.diff(np.concatenate([[0], clk]))
+    assert adv.min() >= 0
+    runs = np.diff(np.concatenate([[-1], np.flatnonzero(adv != 0), [L]])) - 1   # zero-advance run lengths
+    assert runs.max() <= 110, runs.max()
+    for a in range(0, L, 100_000):
+        cpi = (clk[a + 99_999] - (clk[a - 1] if a else 0)) / 100_000
+        assert 0.5 < cpi < 4.0, (a, cpi)
+        assert 5 < k[a:a + 100_000].mean() < 80, (a, k[a:a + 100_000].mean())
