@@ -21,8 +21,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-LIB = os.path.join(PKG, "libpsim.so")
-BUILD = os.path.join(PKG, "_build")
+LIB = os.environ.get("PSIM_LIB_OUT", os.path.join(PKG, "libpsim.so"))   # variant builds (experiments) elsewhere
+BUILD = os.environ.get("PSIM_BUILD_DIR", os.path.join(PKG, "_build"))
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-I", INCLUDE, "-I", CSRC,
