@@ -23,10 +23,11 @@
 // into TMEM, and the epilogue of conv2 position 0), warps 4..7 = EG-B (conv2
 // position 1 -> A3 in TMEM, conv3 epilogue -> a4 rows, staged in smem and stored
 // coalesced), warp 8 = TMEM allocator and MMA issuer (the whole warp runs the loop,
-// one elected lane issues; it also streams W3), warps 9..11 = row builders (block
-// entry {id, k, ws, Clock} -> queue entries -> row indices + time features, staged
-// by cp.async), warps 12..19 = TMA row issuers (trace rows by tile::gather4 straight
-// into the SWIZZLE_128B X tile, evict_first; time features from the row ring).
+// one elected lane issues; it also streams W3), warps 9..11 idle, warps 12..19 = row
+// builders + TMA row issuers (each lane builds one input row per item: block entry
+// {id, k, ws, Clock} -> queue entry -> trace row index + time features, software-
+// pipelined in registers; trace rows by tile::gather4 straight into the SWIZZLE_128B X
+// tile, evict_first).
 // W1/W2 stay resident in smem (48 KB); W3 (64 KB) is streamed one K-half (32 KB) at
 // a time from L2, alternating with the conv3 MMAs.  Per 128-block tile the MMA
 // order is
@@ -50,13 +51,8 @@ constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of
 constexpr int NX = 3;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
 constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][128 B] (half rows)
-// gather metadata staged by cp.async (no register waits on loads in flight):
-constexpr int SMETA_OFF = STG_OFF + 16 * 1024;   // uint4 [4 tiles][128] block entries {id, k, ws lo, Clock lo}
-constexpr int SENT_OFF = SMETA_OFF + 8192;   // uint4 [3 items][128][2] queue entries of rows 2j, 2j+1 (item n in slot n % 3)
-constexpr int RQ = 3;                        // row ring: items built ahead of the TMA issue
-constexpr int RROW_OFF = SENT_OFF + 3 * 4096; // u32   [RQ][2][128] trace16 row of input row 2j+h of block m
-constexpr int RT_OFF = RROW_OFF + RQ * 1024; // uint2 [RQ][2][128] its time-feature chunk
-constexpr int BAR_OFF = RT_OFF + RQ * 2048;  // mbarriers
+constexpr int BE_OFF = STG_OFF + 16 * 1024;  // uint4 [3 tiles][256 issuer lanes]: block entries staged by cp.async
+constexpr int BAR_OFF = BE_OFF + 12 * 1024;  // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 static_assert(SMEM <= 232448, "conv_stack smem over the 227 KB opt-in limit");
@@ -66,13 +62,15 @@ static_assert(SMEM <= 232448, "conv_stack smem over the 227 KB opt-in limit");
 // from TMEM: no smem traffic for A2 / A3.
 constexpr int TMEM_C1 = 0, TMEM_C2 = 128, TMEM_C3 = 384, TMEM_COLS = 512;
 // warps 0-3 EG-A (conv1 epi + conv2 position 0 epi), 4-7 EG-B (conv2 position 1 + conv3
-// epi + a4 stores), 8 MMA + W3 stream, 9-11 row builders, 12-19 TMA row issuers (8 warps x
+// epi + a4 stores), 8 MMA + W3 stream, 9-11 idle, 12-19 row builders + TMA row issuers (8 warps x
 // 8 lanes: the gather4 issue rate scales with issuing warps).  Five warpgroups; registers
 // rebalanced with setmaxnreg (each SM sub-partition holds one warp of every warpgroup):
-// EG-A 136 + EG-B 136 + MMA/builders 96 + issuers 56 + 56 = 480 <= 512.
+// EG-A 136 + EG-B 136 + MMA 96 + issuers 56 + 56 = 480 (= the launch allocation, 96 per thread:
+// setmaxnreg only moves registers between the warps of a CTA; a larger sum deadlocks the inc).
 constexpr int THREADS = 640;
-constexpr int MMA_WARP = 8, BUILD_WARP0 = 9, NBUILD = 3, GATHER_WARP0 = 12, NISSUE = 8;
-constexpr int REG_EPI = 136, REG_ISSUE = 56;
+constexpr int MMA_WARP = 8, GATHER_WARP0 = 12, NISSUE = 8;
+constexpr int REG_EPI = 136, REG_MMA = 96, REG_ISSUE = 56;   // 136 + 136 + 96 + 56 + 56 = 480 = 640 x 96 / 128
+static_assert(2 * REG_EPI + REG_MMA + 2 * REG_ISSUE <= THREADS * 96 / 128, "setmaxnreg over the CTA's allocation");
 
 }  // namespace cs
 
@@ -176,15 +174,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
-  uint64_t* rfull = bars + 32;     // [RQ] 2 builder warps: rows of the item in the ring
-  uint64_t* rempty = bars + 36;    // [RQ] 4 issuer warps: ring slot consumed
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 44);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (tid == 0) {
     for (int i = 0; i < cs::NX; ++i) { mbar_init(xfull + i, cs::NISSUE); mbar_init(xempty + i, 1); }
-    for (int i = 0; i < cs::RQ; ++i) { mbar_init(rfull + i, cs::NBUILD); mbar_init(rempty + i, cs::NISSUE); }
     for (int i = 0; i < 2; ++i) {
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 1); mbar_init(a2full + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 1); mbar_init(a3full + i, 4);
@@ -218,6 +213,12 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
   if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
   if (warp <= cs::MMA_WARP) mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
+  // register budget (setmaxnreg redistributes the launch allocation of 640 x 96; with
+  // REG_MMA < 96 the MMA warpgroup would release registers to the issuers -- measured:
+  // ptxas then spills in the MMA loop, so it stays at the launch value)
+  if constexpr (cs::REG_MMA < 96) {
+    if (warp >= cs::MMA_WARP && warp < cs::GATHER_WARP0) setmaxnreg_dec<cs::REG_MMA>();
+  }
   const float* sb1 = reinterpret_cast<const float*>(sm + cs::BIAS_OFF);
   const float* sb2 = sb1 + 64;
   const float* sb3 = sb1 + 192;
@@ -315,8 +316,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     __syncwarp();
   } else if (warp < 4) {   // ============ EG-A: conv1 epilogues (C1 -> A2, in TMEM) + conv2 position 0 epilogue
     setmaxnreg_inc<cs::REG_EPI>();
-    const int q = warp & 3;
-    const int m = q * 32 + lane;                    // tile row = TMEM lane
+    const int q = warp & 3;                         // TMEM lane quadrant (tile rows 32 q .. 32 q + 31)
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t it = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
@@ -419,39 +419,111 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       prev_tl = tl;
     }
     if (it > 0) e3(it - 1, prev_tl);
-  } else if (warp >= cs::GATHER_WARP0) {   // ============================ TMA row issuers (warps 12..19)
+  } else if (warp >= cs::GATHER_WARP0) {   // ============================ row builders + TMA issuers (warps 12..19)
     // Operand row layout (per input row, 64 bf16): cols 0..46 the trace attributes,
-    // col 47 zero, cols 48..50 the time features, cols 51..63 zero.  The 96-B rows are
-    // fetched by the TMA unit with tile::gather4 (4 arbitrary trace16 rows per
-    // instruction, SWIZZLE_128B applied on the way) into chunks 0..5: issuer warp wq
-    // covers blocks 16 wq .. 16 wq + 15 (lanes 0..7: gather4 of blocks 16 wq + 4 g .. + 3,
-    // atom h); lane l writes chunk 6 (time features) of block 16 wq + (l & 15), atom l >> 4;
-    // chunk 7 is zeroed once.  Each warp arrives on the slot's xfull barrier with the byte
-    // count its gathers deliver (expect_tx), so xfull completes when the last row lands.
+    // col 47 zero, cols 48..50 the time features, cols 51..63 zero.  Item n = conv1
+    // position j = n % 4 of this CTA's tile n / 4: input rows R = 8p + 2j + h (h = 0, 1;
+    // PAPER.md:93 row order) of the tile's 128 blocks (b, p).
+    // Lane l of issuer warp wq BUILDS the row of block m = 16 wq + (l & 15), h = l >> 4:
+    // padding (R > k) -> the all-zero trace16 row past the rank's rows; R = 0 -> the
+    // current instruction; context rows newest first -> the row of queue entry k - R (R6),
+    // with the time features age / remaining-to-complete / remaining-to-retire (R2) in
+    // chunk 6 (cols 48..55) of its SW128 operand row.  The metadata chain block entry
+    // {b << 4 | p, k, ws, Clock} -> queue entry is software-pipelined in registers: the
+    // block entries of tile T + 1 are loaded at the start of tile T and the queue entries
+    // of item n + 2 after item n is issued (L2-only loads, .cg), so no load latency sits
+    // on the issue path.  Lanes 0..7 then ISSUE the rows by TMA tile::gather4 (4 arbitrary
+    // 96-B trace16 rows per instruction, SWIZZLE_128B applied on the way) into chunks 0..5
+    // of the X slot: lane (g, h) = (l & 3, l >> 2 & 1) fetches blocks 16 wq + 4 g .. + 3,
+    // atom h, with the row indices shuffled from the building lanes.  Each warp arrives on
+    // the slot's xfull barrier with the byte count its gathers deliver (expect_tx), so
+    // xfull completes when the last row lands.
     setmaxnreg_dec<cs::REG_ISSUE>();
     const int wq = warp - cs::GATHER_WARP0;          // issuer warp 0..7
     const int m = 16 * wq + (lane & 15), hh = lane >> 4;
-    const uint32_t* rRow = reinterpret_cast<const uint32_t*>(sm + cs::RROW_OFF);
-    const uint2* rT = reinterpret_cast<const uint2*>(sm + cs::RT_OFF);
 #pragma unroll
     for (int s2 = 0; s2 < cs::NX; ++s2) st_sw128(sm + cs::X_OFF + s2 * 32768 + hh * 16384, m, 7, make_uint4(0, 0, 0, 0));
     const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    const uint32_t n_items = my_tiles * 4;
-    const int g = lane & 3, h = (lane >> 2) & 1;     // lane l < 8: rows of atom h, blocks 16 wq + 4 g .. + 3
-    // trace rows are streamed through L2 with evict_first (PSIM_ROW_EVICT=0: normal): the
-    // step's context rows (~145 MB at config 3, G = 1) exceed L2 and would otherwise push
-    // out the queue entries, states and a4 rows that are reused within the step
+    const int g = lane & 3, h = (lane >> 2) & 1;     // TMA lane l < 8: rows of atom h, blocks 16 wq + 4 g .. + 3
+    // trace rows are streamed through L2 with evict_first: the step's context rows
+    // (~145 MB at config 3, G = 1) exceed L2 and would otherwise push out the queue
+    // entries, states and a4 rows that are reused within the step
     const uint64_t pol = l2_policy_evict_first();
-#pragma unroll 1
-    for (uint32_t nI = 0; nI < n_items; ++nI) {
-      const uint32_t it = nI >> 2;   // tile (timestamps only)
-      const int j = (int)(nI & 3);
+    const uint4 kNoBlock = make_uint4(0xFFFFFFFFu, 0u, 0u, 0u);
+    auto row_R = [&](const uint4& be, uint32_t n) -> int { return (int)(be.x & 15) * 8 + 2 * (int)(n & 3) + hh; };
+    auto load_entry = [&](const uint4& be, uint32_t n) -> uint4 {   // queue entry of this lane's row of item n
+      const int R = row_R(be, n), k = (int)be.y;
+      if (be.x == 0xFFFFFFFFu || R < 1 || R > k) return make_uint4(0, 0, 0, 0);
+      return __ldcg(a.q + (uint64_t)(k - R) * a.qn + (be.x >> 4));
+    };
+    // Metadata pipeline: block entries of tiles T and T + 1 in registers (from smem); the
+    // queue entry of item n + 4 is prefetched into L2 (no register) and loaded into
+    // registers at item n + 2 (evA / evB by item parity), so neither the DRAM nor the L2
+    // latency of the step's loaded memory system sits on the issue path.  The loop is
+    // unrolled by two so a pending load is never the source of a register move (a move
+    // would wait for the load).
+    // block entries of tile T live in smem slot T % 3 (lane-private), staged by cp.async two
+    // tiles ahead; beC / beN are register copies of tiles T / T + 1 read at each tile start
+    uint4* sBE = reinterpret_cast<uint4*>(sm + cs::BE_OFF) + wq * 32 + lane;
+    auto stage_block = [&](uint32_t T) {
+      const uint32_t bi = (blockIdx.x + T * gridDim.x) * cs::TILE + m;
+      uint4* dst = sBE + (T % 3) * 256;
+      if (T < my_tiles && bi < nblocks) cp_async16(dst, a.blocks + bi);
+      else *dst = kNoBlock;
+      cp_async_commit();
+    };
+    stage_block(0);
+    stage_block(1);
+    cp_async_wait<0>();
+    uint4 beC = sBE[0], beN = sBE[256];
+    stage_block(2);
+    const uint32_t n_items = my_tiles * 4;
+    auto entry_ptr = [&](const uint4& be, uint32_t n) -> const uint4* {   // nullptr: no queue entry
+      const int R = row_R(be, n), k = (int)be.y;
+      if (be.x == 0xFFFFFFFFu || R < 1 || R > k) return nullptr;
+      return a.q + (uint64_t)(k - R) * a.qn + (be.x >> 4);
+    };
+    constexpr bool kPrefetchL2 = false;   // L2 prefetch of item n + 4's entry: measured slower (LSU pressure)
+#pragma unroll
+    for (uint32_t n = 2; n < 4; ++n)
+      if (kPrefetchL2)
+        if (const uint4* p = entry_ptr(beC, n)) prefetch_l2(p);
+    uint4 evA = load_entry(beC, 0), evB = load_entry(beC, 1);
+    auto item = [&](uint32_t nI, uint4& ev) {
+      const uint32_t it = nI >> 2;                     // this CTA's tile of item nI
+      [[maybe_unused]] const int j = (int)(nI & 3);    // conv1 position (timestamps)
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
-      const int rs = (int)(nI % cs::RQ);
-      wait_full(rfull + rs, nI / cs::RQ);
+      // ---- build this lane's row of item nI
+      uint32_t row;
+      uint2 tc = make_uint2(0u, 0u);
+      {
+        const int R = row_R(beC, nI), k = (int)beC.y;
+        if (beC.x == 0xFFFFFFFFu || R > k) {
+          row = a.zero_row;                                        // zero padding at the tail
+        } else if (R == 0) {
+          row = (uint32_t)((int64_t)(beC.z + (uint32_t)a.step) - a.row_lo);   // current instruction first
+        } else {
+          const int c = ev.z & 0xFFFF, sv = (ev.z >> 16) & 0xFFFF;
+          const int age = (int)(beC.w - ev.y);
+          const int t0 = min(age, kTimeMax), t1 = min(max(0, c - age), kTimeMax), t2 = min(c + sv - age, kTimeMax);
+          tc = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
+          row = (uint32_t)((int64_t)ev.x - a.row_lo);
+        }
+      }
+      if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
+      // the entry of item nI + 2 (tile it or it + 1) into the same registers; item nI + 4
+      // (tile it + 1) into L2
+      const uint32_t n2 = nI + 2;
+      ev = (n2 < n_items) ? load_entry((n2 >> 2) == it ? beC : beN, n2) : make_uint4(0, 0, 0, 0);
+      if (kPrefetchL2 && nI + 4 < n_items)
+        if (const uint4* p = entry_ptr(beN, nI + 4)) prefetch_l2(p);
+      if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
+      // row indices of the 4 blocks this lane gathers (TMA lanes 0..7): lanes 4 g + i + 16 h
+      const uint32_t r0 = __shfl_sync(0xffffffffu, row, 4 * g + 0 + 16 * h);
+      const uint32_t r1 = __shfl_sync(0xffffffffu, row, 4 * g + 1 + 16 * h);
+      const uint32_t r2 = __shfl_sync(0xffffffffu, row, 4 * g + 2 + 16 * h);
+      const uint32_t r3 = __shfl_sync(0xffffffffu, row, 4 * g + 3 + 16 * h);
       if (warp == cs::GATHER_WARP0) PSIM_TS(104 + j);
-      const uint2 tc = rT[(rs * 2 + hh) * 128 + m];
-      const uint4 r4 = *reinterpret_cast<const uint4*>(rRow + (rs * 2 + h) * 128 + 16 * wq + 4 * g);
       const int xs = (int)(nI % cs::NX);
       wait_empty(xempty + xs, nI / cs::NX);
       if (warp == cs::GATHER_WARP0) PSIM_TS(82 + 3 * j);
@@ -459,118 +531,29 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       // chunk 6 (cols 48..55): time features of context rows, zero otherwise (R2); the TMA
       // writes only chunks 0..5, so this can go in before the rows land
       st_sw128(xa + hh * 16384, m, 6, make_uint4(tc.x, tc.y, 0u, 0u));
+      if (warp == cs::GATHER_WARP0) PSIM_TS(112 + 3 * j);
       fence_async_smem();                               // chunk 6 visible to tcgen05
       __syncwarp();
+      if (warp == cs::GATHER_WARP0) PSIM_TS(113 + 3 * j);
       if (lane == 0) mbar_expect_tx(xfull + xs, 32 * 96);   // arrive + this warp's 32 rows of 96 B
       __syncwarp();
+      if (warp == cs::GATHER_WARP0) PSIM_TS(114 + 3 * j);
       if (lane < 8)
-        tma_gather4_hint(xa + h * 16384 + (16 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r4.x, r4.y, r4.z, r4.w, pol);
+        tma_gather4_hint(xa + h * 16384 + (16 * wq + 4 * g) * 128, &tmX, xfull + xs, 0, r0, r1, r2, r3, pol);
       __syncwarp();
-      if (lane == 0) mbar_arrive(rempty + rs);          // ring slot consumed (its values are in registers)
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
-    }
-  } else {   // ============================ row builders (warps 9..11)
-    // Builder thread tb owns blocks tb and tb + 96 (< 128) of each tile and computes, for every
-    // item (conv1 position j), the trace16 rows of their input rows 2j and 2j+1 and the
-    // time-feature chunks (cols 48..55: age, remaining-to-complete, remaining-to-retire of
-    // context rows, R2; zero otherwise) into the row ring, RQ items ahead of the TMA issue.
-    // Rows: padding -> the all-zero row past the rank's rows, R = 0 -> the current
-    // instruction, context rows newest first -> the row of queue entry k - R (R6).
-    //
-    // The metadata chain block entry (id + the sub-trace state, written with the id by
-    // the previous step's update) -> queue entries is staged in shared memory by
-    // cp.async, so no register ever waits on a load in flight: iteration n (tile t,
-    // item j) issues the block entries of tile t+2 (j == 0) and the queue entries of
-    // item n+2, and consumes what iterations <= n-2 staged (cp.async.wait_group 1: one
-    // group per iteration).
-    const int tb = (warp - cs::BUILD_WARP0) * 32 + lane;   // 0..95: blocks tb and tb + 96 (< 128)
-    constexpr int NB = cs::NBUILD * 32;
-    uint4* sMeta = reinterpret_cast<uint4*>(sm + cs::SMETA_OFF);
-    uint4* sEnt = reinterpret_cast<uint4*>(sm + cs::SENT_OFF);
-    uint32_t* rRow = reinterpret_cast<uint32_t*>(sm + cs::RROW_OFF);
-    uint2* rT = reinterpret_cast<uint2*>(sm + cs::RT_OFF);
-    const uint32_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    const uint32_t n_items = my_tiles * 4;
-    auto valid_of = [&](uint32_t T, int m) -> bool {   // block m of this CTA's T-th tile exists
-      const uint32_t tl = blockIdx.x + T * gridDim.x;
-      return T < my_tiles && tl * cs::TILE + m < nblocks;
-    };
-    auto stage_meta = [&](uint32_t T) {                // stage 1: block entries {id, k, ws lo, Clock lo} of tile T
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int m = tb + NB * u;
-        if (m < cs::TILE && valid_of(T, m))
-          cp_async16(sMeta + (T & 3) * 128 + m, a.blocks + (blockIdx.x + T * gridDim.x) * cs::TILE + m);
+      if (((nI + 1) & 3) == 0) {                        // the next item starts tile it + 1
+        cp_async_wait<0>();                             // tile it + 2's entries (staged a tile ago)
+        beC = beN;
+        beN = sBE[((it + 2) % 3) * 256];
+        stage_block(it + 3);                            // into slot it % 3 (tile it is done)
       }
     };
-    auto stage_ent = [&](uint32_t n) {                 // stage 2: queue entries of item n (block entries landed)
-      const uint32_t T = n >> 2;
-      const int j = (int)(n & 3);
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int m = tb + NB * u;
-        if (m >= cs::TILE || !valid_of(T, m)) continue;
-        const uint4 mt = sMeta[(T & 3) * 128 + m];
-        const int k = (int)mt.y;
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int R = (int)(mt.x & 15) * 8 + 2 * j + h;   // input row (PAPER.md:93 row order)
-          if (R >= 1 && R <= k)                              // context row: entry k - R (newest first, R6)
-            cp_async16(sEnt + ((n % 3) * 128 + m) * 2 + h, a.q + (uint64_t)(k - R) * a.qn + (mt.x >> 4));
-        }
-      }
-    };
-    auto row_of = [&](bool valid, const uint4& mt, int R, const uint4& ev, uint2& tchunk) -> uint32_t {
-      tchunk = make_uint2(0u, 0u);
-      const int k = (int)mt.y;
-      if (!valid || R > k) return a.zero_row;                 // zero padding at the tail
-      if (R == 0) return (uint32_t)((int64_t)(mt.z + (uint32_t)a.step) - a.row_lo);   // current first
-      const int c = ev.z & 0xFFFF, sv = (ev.z >> 16) & 0xFFFF;
-      const int age = (int)(mt.w - ev.y);
-      const int t0 = min(age, kTimeMax), t1 = min(max(0, c - age), kTimeMax), t2 = min(c + sv - age, kTimeMax);
-      tchunk = make_uint2(pack_bf16((float)t0, (float)t1), pack_bf16((float)t2, 0.f));
-      return (uint32_t)((int64_t)ev.x - a.row_lo);
-    };
-    // prologue: block entries of tiles 0..1, queue entries of items 0..1
-    for (uint32_t T = 0; T < 2; ++T) stage_meta(T);
-    cp_async_commit();
-    cp_async_wait<0>();
-    stage_ent(0);
-    stage_ent(1);
-    cp_async_commit();
-    cp_async_commit();   // two groups so that wait_group 1 at item 0 covers the entries of item 0
 #pragma unroll 1
-    for (uint32_t nI = 0; nI < n_items; ++nI) {
-      const uint32_t it = nI >> 2;
-      const int j = (int)(nI & 3);
-      if (warp == cs::BUILD_WARP0) PSIM_TS(112 + 3 * j);
-      cp_async_wait<1>();                             // everything staged up to iteration nI - 2 has landed
-      if (warp == cs::BUILD_WARP0) PSIM_TS(113 + 3 * j);
-      const int rs = (int)(nI % cs::RQ);
-      wait_empty(rempty + rs, nI / cs::RQ);
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int m = tb + NB * u;
-        if (m >= cs::TILE) continue;
-        const bool valid = valid_of(it, m);
-        const uint4 mt = sMeta[(it & 3) * 128 + m];
-        const uint4 e0 = sEnt[((nI % 3) * 128 + m) * 2], e1 = sEnt[((nI % 3) * 128 + m) * 2 + 1];
-        const int R0 = (int)(mt.x & 15) * 8 + 2 * j;
-        uint2 tA, tB;
-        rRow[(rs * 2 + 0) * 128 + m] = row_of(valid, mt, R0, e0, tA);
-        rRow[(rs * 2 + 1) * 128 + m] = row_of(valid, mt, R0 + 1, e1, tB);
-        rT[(rs * 2 + 0) * 128 + m] = tA;
-        rT[(rs * 2 + 1) * 128 + m] = tB;
-      }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(rfull + rs);
-      if (warp == cs::BUILD_WARP0) PSIM_TS(114 + 3 * j);
-      // stage the metadata of later iterations
-      if (j == 0) stage_meta(it + 2);
-      if (nI + 2 < n_items) stage_ent(nI + 2);
-      cp_async_commit();
+    for (uint32_t nI = 0; nI < n_items; nI += 2) {      // n_items is a multiple of 4
+      item(nI, evA);
+      item(nI + 1, evB);
     }
-    cp_async_wait<0>();
   }
   fence_before();
   __syncthreads();

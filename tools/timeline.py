@@ -20,11 +20,11 @@ for h in range(2):
     names[59 + 4 * h] = f"e2({h})done"
 names.update({64: "e3wait", 65: "e3C3", 66: "e3done", 67: "e3staged", 68: "e3ld0", 69: "e3ld1", 80: "g start"})
 for j in range(4):
-    names[81 + 3 * j] = f"g{j}a"; names[82 + 3 * j] = f"g{j}slot"; names[83 + 3 * j] = f"g{j}xfull(prev)"
+    names[81 + 3 * j] = f"g{j}a"; names[82 + 3 * j] = f"g{j}slot"; names[83 + 3 * j] = f"g{j}built"
 for j in range(4):
-    names[96 + 2 * j] = f"g{j}issued"; names[97 + 2 * j] = f"g{j}staged"
+    names[96 + 2 * j] = f"g{j}issued"; names[97 + 2 * j] = f"g{j}ldq"
     names[104 + j] = f"g{j}rfull"
-    names[112 + 3 * j] = f"b{j}top"; names[113 + 3 * j] = f"b{j}staged"; names[114 + 3 * j] = f"b{j}built"
+    names[112 + 3 * j] = f"g{j}sts"; names[113 + 3 * j] = f"g{j}fenced"; names[114 + 3 * j] = f"g{j}expect"
 names.update({128: "tma start", 129: "tma end", 132: "mma wait tempty", 133: "mma start", 134: "mma issued",
               140: "epi start", 141: "epi F ready", 142: "epi y done", 145: "upd start", 146: "upd y ready",
               143: "upd done", 144: "upd scan"})
