@@ -199,12 +199,12 @@ def ncu_traffic(kernel_class):
 
 
 # --------------------------------------------------------------------------- CPU oracle
-def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None, seed=7):
+def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None, seed=7, sparse=False):
     """Run the oracle (as it stands, single thread) on whole sub-traces of the same
     workload until ~budget_s of CPU time; returns (instructions, seconds, cycles)."""
     import oracle
     import synth
-    w = synth.weights(cfg["arch"])
+    w = synth.weights(cfg["arch"], sparse24=sparse)
     mode = oracle.BF16 if cfg["precision"] == "bf16" else oracle.FP64
     rng = np.random.default_rng(seed)
     done, t_used, per = 0, 0.0, {}
@@ -235,10 +235,10 @@ def oracle_sample(cfg, tr_rows, row_lo, budget_s, L, N, W, j_list=None, seed=7):
 
 def _oracle_worker(args):
     """One all-core oracle process: whole random sub-traces for ~budget_s of its own CPU."""
-    cfg_name, budget_s, seed = args
+    cfg_name, budget_s, seed, sparse = args
     cfg = CONFIGS[cfg_name]
     os.environ.setdefault("OMP_NUM_THREADS", "1")
-    n_i, t, per = oracle_sample(cfg, None, 0, budget_s, cfg["L"], cfg["N"], cfg["W"], seed=seed)
+    n_i, t, per = oracle_sample(cfg, None, 0, budget_s, cfg["L"], cfg["N"], cfg["W"], seed=seed, sparse=sparse)
     return n_i, t, len(per)
 
 
@@ -256,7 +256,7 @@ def host_info():
     return info
 
 
-def oracle_all_cores(cfg_name, budget_s):
+def oracle_all_cores(cfg_name, budget_s, sparse=False):
     """The oracle as it stands on every host core: P = nproc independent processes, each
     simulating whole random sub-traces of the same workload for ~budget_s.  Returns
     (instructions, wall seconds, P, sub-traces)."""
@@ -265,7 +265,7 @@ def oracle_all_cores(cfg_name, budget_s):
     ctx = mp.get_context("spawn")
     t0 = time.perf_counter()
     with ctx.Pool(P) as pool:
-        res = pool.map(_oracle_worker, [(cfg_name, budget_s, 1000 + i) for i in range(P)])
+        res = pool.map(_oracle_worker, [(cfg_name, budget_s, 1000 + i, sparse) for i in range(P)])
     wall = time.perf_counter() - t0
     # per-process throughput is measured on its own clock; aggregate = sum of per-process rates
     rate = sum(n / t for n, t, _ in res if t > 0)
@@ -288,6 +288,11 @@ def main():
     ap.add_argument("--emulate-rank", default=None, metavar="R/G",
                     help="diagnostics: run rank R's share of a G-GPU job on this one GPU (no NCCL), "
                          "to estimate per-GPU throughput at G GPUs; value = that rank's instructions/s")
+    ap.add_argument("--sparse", action="store_true",
+                    help="2:4 structured sparsity (PAPER.md:157): 2:4-pruned weights on the sparse tcgen05.mma.sp "
+                         "layer-wise path (PSIM_SPARSE24)")
+    ap.add_argument("--layerwise", action="store_true",
+                    help="run the layer-by-layer tcgen05 GEMM path instead of the fused kernels (A/B)")
     ap.add_argument("--correction", type=int, default=0,
                     help="post-error correction limit (PAPER.md:203-219; the paper uses 100); 0 = off")
     args = ap.parse_args()
@@ -316,6 +321,10 @@ def main():
               "queue_rows": 111, "precision": cfg["precision"],
               "l2": "inputs larger than L2 (trace %.1f GB resident in HBM)" % (L * 48 / 1e9),
               "post_error_correction": args.correction}
+    if args.sparse:
+        config["sparsity"] = "2:4 magnitude-pruned tensor-core layers, tcgen05.mma.sp layer-wise path (R22)"
+    if args.layerwise:
+        config["path"] = "layer-wise tcgen05 GEMMs"
 
     if args.impl == "reference":
         # the oracle as it stands, on rank 0 only, on the host cores
@@ -331,7 +340,7 @@ def main():
         with mp.get_context("spawn").Pool(P) as pool:
             for it in range(args.warmup + args.steps):
                 t0 = time.perf_counter()
-                res = pool.map(_oracle_worker, [(args.config, per_step, 100000 * it + i) for i in range(P)])
+                res = pool.map(_oracle_worker, [(args.config, per_step, 100000 * it + i, args.sparse) for i in range(P)])
                 dt = time.perf_counter() - t0
                 if it >= args.warmup:
                     times.append(dt); insts += sum(r[0] for r in res); subs += sum(r[2] for r in res)
@@ -372,7 +381,7 @@ def main():
     host = torch.empty((rows, 48), dtype=torch.uint8, pin_memory=True)
     synth.trace_into(host.numpy(), synth.TRACE_SEED_BASE + cfg["seed_off"], rr.row_lo)
     dev = host.cuda()
-    w = synth.weights(cfg["arch"])
+    w = synth.weights(cfg["arch"], sparse24=args.sparse)
     log(f"[rank {rank}] trace rows [{rr.row_lo},{rr.row_hi}) generated in {time.time() - t0:.1f}s")
 
     stream = torch.cuda.Stream()
@@ -392,7 +401,7 @@ def main():
     sim = P.Simulator(device=local_rank, precision=cfg["precision"], rank=emu[0] if emu else rank,
                       world_size=emu[1] if emu else world, nccl_id=nccl_id,
                       stream=stream.cuda_stream, profile=os.environ.get("PSIM_NOPROF") is None, chunk_steps=int(os.environ.get("PSIM_CHUNK", "0")),
-                      correction_limit=args.correction)
+                      correction_limit=args.correction, sparse24=args.sparse, layerwise=args.layerwise)
     sim.load_model(cfg["arch"], w)
 
     def timed(trace_tensor, k_steps, warm):
@@ -445,10 +454,10 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu:
         # cpu_baseline: the oracle as it stands on a bounded sample of the same workload,
         # plus the sampled sub-traces' cycles vs the GPU (parity sample)
-        n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W)
+        n_i, t, per = oracle_sample(cfg, host.numpy(), rr.row_lo, args.cpu_budget, L, N, W, sparse=args.sparse)
         gcyc = sim.corrections()[1] if args.correction else sim.subtrace_cycles()   # first-pass cycles
         errs = [abs(int(gcyc[j]) - c) / max(c, 1) for j, c in per.items()]
-        n_all, wall_all, P_all, sub_all, rate_all = oracle_all_cores(args.config, args.cpu_budget_all)
+        n_all, wall_all, P_all, sub_all, rate_all = oracle_all_cores(args.config, args.cpu_budget_all, args.sparse)
         line["cpu_baseline"] = {"value": rate_all / 1e6, "unit": "MIPS", "cores": P_all, "kind": "oracle",
                                 "sample": f"all host cores: {P_all} oracle processes x ~{args.cpu_budget_all:.0f} s, "
                                           f"{sub_all} whole random sub-traces ({n_all} counted instructions, W={W} "

@@ -61,6 +61,16 @@ extern "C" {
                                 given trajectory, R17)                              */
 #define PSIM_LAYERWISE 8u    /* bf16 C3: use the layer-by-layer GEMM path instead of the fused
                                 padding-aware kernels (A/B comparison, parity of both)       */
+#define PSIM_SPARSE24 16u    /* 2:4 structured sparsity (PAPER.md:157 [IV-B], :261 [VI-B]): the
+                                model's tensor-core layers (C3 / M2 conv1..3 and fc1, bf16) must be
+                                2:4 sparse along their reduction dimension K in the device order
+                                (conv: K = tap * Cin_dev + channel, groups of 4 consecutive input
+                                channels of one tap; fc1: 4 consecutive flattened inputs) -- e.g.
+                                magnitude-pruned weights, which the oracle loads unchanged; they are
+                                compressed at psim_load_model and every layer runs on the sparse
+                                tcgen05.mma.sp GEMM of the layer-wise path.  load_model returns ARG
+                                if a group holds more than 2 nonzeros, UNSUPPORTED for other
+                                architectures or fp32                                          */
 #define PSIM_PROFILE 2u      /* time kernel classes with CUDA events on the launch stream: every
                                 launch outside the step loop and the launches of every 16th
                                 lockstep step (events between all launches would serialise the

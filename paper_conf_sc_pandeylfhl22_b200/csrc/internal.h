@@ -37,6 +37,11 @@ struct GemmLayer {
   void* w = nullptr;       // device [N][K], fp32 or bf16 (K-major)
   float* bias = nullptr;   // device [N] fp32
   void* w_tc = nullptr;    // device weights pre-tiled for the tcgen05 kernel (bf16)
+  // 2:4 structured sparsity (PSIM_SPARSE24, R22): compressed weights [sp_mh*128][K/2]
+  // bf16 and the tcgen05.mma.sp metadata words [sp_mh * K/32][128] (gemm_sp.cu)
+  void* w_sp = nullptr;
+  uint32_t* meta = nullptr;
+  int sp_mh = 0;
 };
 
 struct Model {
@@ -177,6 +182,13 @@ bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(const __nv_bfloat16* A, const void* Wtc, const float* b, void* C,
                     bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st, int taps = 1,
                     const __nv_bfloat16* resid = nullptr, int pad_period = 0);
+// 2:4 sparse layer (gemm_sp.cu): W bf16 [N][K] (host, RNE bits) -> compressed [mh*128][K/2]
+// and metadata words; 0 on success, -1 unsupported shape, -2 not 2:4 sparse along K
+int sparse24_compress(const uint16_t* W, int N, int K, std::vector<uint16_t>* wc, std::vector<uint32_t>* meta,
+                      int* mh);
+// C[M][N] = act(X[M][K] . W^T + b) with W 2:4-sparse (compressed + metadata from sparse24_compress)
+void launch_gemm_sp(const __nv_bfloat16* X, const __nv_bfloat16* Wc, const uint32_t* meta, int mh, const float* b,
+                    void* C, bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st);
 // Pre-tile a [N][K] bf16 weight for the tensor-core kernel (device -> device).
 void* pretile_weight_tc(const __nv_bfloat16* W, int N, int K, cudaStream_t st);
 

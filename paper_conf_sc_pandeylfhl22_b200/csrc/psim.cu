@@ -252,7 +252,7 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->d_forced);
   for (auto e : ctx->ld_events) cudaEventDestroy(e);
   if (ctx->ld_stream) cudaStreamDestroy(ctx->ld_stream);
-  for (auto& l : ctx->model.layers) { dfree(l.w); dfree(l.bias); }
+  for (auto& l : ctx->model.layers) { dfree(l.w); dfree(l.bias); dfree(l.w_sp); dfree(l.meta); }
   dfree(ctx->model.head_w);
   dfree(ctx->model.head_b);
   SimState& s = ctx->st;
@@ -406,13 +406,16 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
     ls.push_back({1, 256, 3, 0});
     if (ctx->opts.precision != PSIM_BF16) FAIL(PSIM_ERR_UNSUPPORTED, "RB7 runs on the bf16 tensor-core path only");
   } else FAIL(PSIM_ERR_ARG, "unknown arch %u", desc->arch);
+  const bool sparse = (ctx->opts.flags & PSIM_SPARSE24) != 0;
+  if (sparse && (rb7 || ctx->opts.precision != PSIM_BF16))
+    FAIL(PSIM_ERR_UNSUPPORTED, "PSIM_SPARSE24 needs the bf16 C3 or M2 model");
   uint64_t need = 0;
   for (auto& l : ls) need += (uint64_t)l.cout * l.cin * (l.kind != 1 ? l.k : 1) + l.cout;
   if (need != n_floats) FAIL(PSIM_ERR_ARG, "weight count %llu != %llu for arch %u", (unsigned long long)n_floats,
                              (unsigned long long)need, desc->arch);
   CK(cudaSetDevice(ctx->opts.device));
   Model& m = ctx->model;
-  for (auto& l : m.layers) { dfree(l.w); dfree(l.bias); }
+  for (auto& l : m.layers) { dfree(l.w); dfree(l.bias); dfree(l.w_sp); dfree(l.meta); }
   m.layers.clear();
   dfree(m.head_w); dfree(m.head_b);
   m.head_w = m.head_b = nullptr;
@@ -494,6 +497,17 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
         CK(cudaStreamSynchronize(ctx->stream));
         CK(cudaGetLastError());
       }
+      if (sparse) {   // 2:4 compression + tcgen05.mma.sp metadata (gemm_sp.cu)
+        std::vector<uint16_t> wc;
+        std::vector<uint32_t> meta;
+        const int rc = sparse24_compress(wb.data(), g.N, g.K, &wc, &meta, &g.sp_mh);
+        if (rc == -2) FAIL(PSIM_ERR_ARG, "layer %zu: weights are not 2:4 sparse along K (PSIM_SPARSE24)", li);
+        if (rc != 0) FAIL(PSIM_ERR_UNSUPPORTED, "layer %zu: K = %d, N = %d unsupported by the sparse GEMM", li, g.K, g.N);
+        CK(cudaMalloc(&g.w_sp, wc.size() * 2));
+        CK(cudaMemcpy(g.w_sp, wc.data(), wc.size() * 2, cudaMemcpyHostToDevice));
+        CK(cudaMalloc(&g.meta, meta.size() * 4));
+        CK(cudaMemcpy(g.meta, meta.data(), meta.size() * 4, cudaMemcpyHostToDevice));
+      }
     } else {
       CK(cudaMalloc(&g.w, Wk.size() * 4));
       CK(cudaMemcpy(g.w, Wk.data(), Wk.size() * 4, cudaMemcpyHostToDevice));
@@ -511,7 +525,7 @@ int psim_load_model(psim_ctx* ctx, const psim_model_desc* desc, const float* w, 
   dfree(fz.T);
   fz.T = nullptr;
   fz.ready = false;
-  if (bf16 && desc->arch == PSIM_ARCH_C3) {
+  if (bf16 && desc->arch == PSIM_ARCH_C3 && !sparse) {   // (a 2:4 model runs layer-wise on the sparse GEMM)
     // c3 = conv3(conv2(conv1(0))) with the GPU's rounding points (bf16 operands,
     // bias + ReLU, bf16 activations); T[P] = b_fc1 + sum_{p>=P} Wfc1[:, p*128:(p+1)*128] . c3
     auto bf = [](double v) { uint16_t h = f32_to_bf16_rne((float)v); uint32_t u = (uint32_t)h << 16; float f; memcpy(&f, &u, 4); return (double)f; };
@@ -614,7 +628,10 @@ static int run_cnn(psim_ctx* ctx, uint64_t n) {
     const int64_t M = (int64_t)n * g.rows_per_item;
     if (g.block_begin) block_in = in;
     pf.begin(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
-    if (bf16) {
+    if (bf16 && g.w_sp) {   // 2:4 structured-sparse tcgen05.mma.sp (PSIM_SPARSE24)
+      launch_gemm_sp((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w_sp, g.meta, g.sp_mh, g.bias, out, last, M,
+                     g.N, g.K, g.relu, ctx->stream);
+    } else if (bf16) {
       if (g.taps > 1 || g.add_block_input || g.pad_period) {
         if (!g.w_tc) FAIL(PSIM_ERR_UNSUPPORTED, "layer %zu needs the tensor-core kernel", li);
         launch_gemm_tc((const __nv_bfloat16*)in, g.w_tc, g.bias, out, last, M, g.N, g.K, g.relu, ctx->stream, g.taps,

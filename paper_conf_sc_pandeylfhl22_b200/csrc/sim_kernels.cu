@@ -131,7 +131,10 @@ void launch_mrow(const uint8_t* trace, int64_t stride, int64_t rows, uint8_t* ou
 
 __global__ void state_init_kernel(SimState s) {
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (t < s.n) { s.clock[t] = 0; s.bnd[t] = 0; s.cycles[t] = 0; s.count[t] = 0; }
+  if (t < s.n) {
+    s.clock[t] = 0; s.bnd[t] = 0; s.cycles[t] = 0; s.count[t] = 0;
+    if (s.rmin) s.rmin[t] = 0;   // meaningful only when count > 0; defined for the sanitizer (initcheck)
+  }
   if (t < 112) s.k_hist[t] = 0;
   if (t == 0) { *s.stalls = 0; *s.total = 0; *s.ptile_sum = 0; }
 }

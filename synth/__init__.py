@@ -145,10 +145,38 @@ def calibration(arch: str):
     return np.ones(3), np.zeros(3)
 
 
-def weights(arch: str = "C3", seed: int = WEIGHT_SEED, *, gain=None, bias=None) -> np.ndarray:
-    """Flat fp32 weight vector for ``arch`` (PyTorch layouts, layers in order)."""
+def prune24(w: np.ndarray, kind: str) -> np.ndarray:
+    """2:4 magnitude pruning of one tensor-core layer (R22; the paper prunes its
+    trained model for 2:4 structured sparsity): in every group of 4
+    consecutive inputs along the reduction dimension -- input channels of one conv tap
+    (PyTorch [Cout][Cin][k]: w[o, 4g:4g+4, t]), or 4 consecutive flattened inputs of a
+    linear layer -- keep the 2 largest magnitudes (ties: the lower index), zero the rest.
+    This is model preparation (an input both the oracle and the GPU load unchanged), not
+    part of the simulation."""
+    w = np.array(w, dtype=np.float64, copy=True)
+    if kind == "conv":
+        cout, cin, k = w.shape
+        v = np.moveaxis(w, 2, 1)                      # [Cout][k][Cin]
+    else:
+        cout, cin = w.shape
+        v = w[:, None, :]                             # [Cout][1][Cin]
+    pad = (-cin) % 4
+    vp = np.concatenate([v, np.zeros(v.shape[:2] + (pad,))], axis=2) if pad else v
+    g = vp.reshape(vp.shape[0], vp.shape[1], -1, 4)
+    order = np.argsort(-np.abs(g), axis=3, kind="stable")
+    keep = np.zeros_like(g, dtype=bool)
+    np.put_along_axis(keep, order[..., :2], True, axis=3)
+    g = np.where(keep, g, 0.0)
+    vp = g.reshape(vp.shape)[:, :, :cin]
+    return np.moveaxis(vp, 1, 2) if kind == "conv" else vp[:, 0, :]
+
+
+def weights(arch: str = "C3", seed: int = WEIGHT_SEED, *, gain=None, bias=None, sparse24: bool = False) -> np.ndarray:
+    """Flat fp32 weight vector for ``arch`` (PyTorch layouts, layers in order).  With
+    ``sparse24`` every tensor-core layer (all but the fc2 head) is 2:4 magnitude-pruned
+    (prune24) and the head uses its own calibration entry ``<arch>:24``."""
     if gain is None or bias is None:
-        g0, b0 = calibration(arch)
+        g0, b0 = calibration(arch + (":24" if sparse24 else ""))
         gain = g0 if gain is None else np.asarray(gain, np.float64)
         bias = b0 if bias is None else np.asarray(bias, np.float64)
     parts = []
@@ -161,6 +189,8 @@ def weights(arch: str = "C3", seed: int = WEIGHT_SEED, *, gain=None, bias=None) 
         b = (2.0 * _splitmix_uniform(seed, 2 * li + 1, bs[0]) - 1.0) / np.sqrt(fan_in)
         if li == 0:
             w = w / FEATURE_SCALE[None, :, None]
+        if sparse24 and li < len(shapes) - 1:                # tensor-core layers only (not the fc2 head)
+            w = prune24(w, "conv" if len(ws) == 3 else "linear")
         if li == len(shapes) - 1:                            # calibrated head
             if arch in FLOOR_ARCHS:
                 w[FLOOR_OUTPUT] = np.abs(w[FLOOR_OUTPUT])    # completion row non-negative (R21)

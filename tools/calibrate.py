@@ -37,11 +37,12 @@ def mixed_trace(n_per):
 def main(archs):
     path = os.path.join(os.path.dirname(synth.__file__), "calibration.json")
     cal = json.load(open(path)) if os.path.exists(path) else {}
-    for arch in archs:
+    for name in archs:
+        arch, sparse = name.split(":")[0], name.endswith(":24")   # "<arch>:24" = the 2:4-pruned model
         tr = mixed_trace(N_PER_PHASE[arch])
         gain, bias = np.ones(3), np.zeros(3)
         for it in range(ITERS):
-            w = synth.weights(arch, gain=gain, bias=bias)
+            w = synth.weights(arch, gain=gain, bias=bias, sparse24=sparse)
             r = oracle.simulate(tr, 8, 0, arch=arch, weights=w)
             y = r["y"].astype(np.float64)
             z = (y - bias) / gain                      # head output at gain 1, bias 0
@@ -56,16 +57,16 @@ def main(archs):
             o, b0 = synth.FLOOR_OUTPUT, synth.COMPLETE_BIAS
             if arch not in synth.FLOOR_ARCHS:
                 o = None
-            zf = None if o is None else = (y[:, o] - b0) / g_prev[o]               # non-negative part at gain 1
+            zf = None if o is None else (y[:, o] - b0) / g_prev[o]   # non-negative part at gain 1
             if o is not None:
                 gain[o] = (TARGET_MEAN[o] - b0) / max(zf.mean(), 1e-9) if it == 0 else \
                     g_prev[o] * np.clip((TARGET_MEAN[o] - b0) / max(y[:, o].mean() - b0, 1e-9), 0.5, 2.0) ** 0.5
                 bias[o] = b0
             lat = r["lat"].astype(np.float64)
-            print(f"{arch} it{it}: y mean {y.mean(0).round(3)} std {y.std(0).round(3)} | "
+            print(f"{name} it{it}: y mean {y.mean(0).round(3)} std {y.std(0).round(3)} | "
                   f"lat mean {lat.mean(0).round(3)} | k mean {r['k'].mean():.1f} max {r['k'].max()}"
                   f" | stalls {r['stalls']}", flush=True)
-        cal[arch] = {"gain": gain.tolist(), "bias": bias.tolist(),
+        cal[name] = {"gain": gain.tolist(), "bias": bias.tolist(),
                      "target_mean": TARGET_MEAN.tolist(), "target_std": TARGET_STD.tolist()}
         json.dump(cal, open(path, "w"), indent=1)
 
