@@ -793,13 +793,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       }
       const bool active = inb && a.u.step < nsteps;
       QBatch first;
-      if (active) {
-        load_qbatch(a.u.st, b, kb, first);
-        // the rest of the queue into L2 while the head runs: the retire scan's later batches
-        // then wait on L2, not DRAM (consecutive threads = consecutive sub-traces: coalesced)
-        const uint64_t qn = a.u.st.qn ? a.u.st.qn : a.u.st.n;
-        for (int e = 8; e < kb; ++e) prefetch_l2(a.u.st.q + (uint64_t)e * qn + b);
-      }
+      if (active) load_qbatch(a.u.st, b, kb, first);   // (an L2 prefetch of the rest of the queue here: no gain)
       const int pb = min((kb + 8) >> 3, 14);
       wait_full(yfull + yb, it >> 1);
       if (q == 0) PSIM_TS(146);

@@ -43,7 +43,7 @@ struct SpCfg {
   static constexpr int B_BYTES = 2 * sp::BN * 128; // activations [128][128 logical K] bf16, two SW128 atoms
   static constexpr int STAGE = A_BYTES + B_BYTES;
   static constexpr int STAGES = (192 * 1024) / STAGE;
-  static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
+  static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + 4 * 32 * 33 * 4;   // + epilogue transpose stages
   static constexpr int ACC_COLS = MH * sp::BN;
   static constexpr int NACC = MH == 1 ? 2 : 1;     // double-buffered accumulators when they fit next to the metadata
 };
@@ -149,7 +149,11 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
   } else {   // ---------------- epilogue (warps 2..5): thread = output channel ----------------
+    // D^T lane = output channel, column = row.  Each 32 x 32 block (32 channels of this warp's
+    // quadrant x 32 rows) goes through a per-warp smem stage (fp32, padded rows) so that lane j
+    // then writes row j's 32 channels as contiguous 16-B stores (64 B bf16 / 128 B fp32 per lane).
     const int q = warp & 3;
+    float* stg = reinterpret_cast<float*>(smem + Cfg::STAGES * Cfg::STAGE + 256) + (warp - 2) * 32 * 33;
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
       const int acc = it % Cfg::NACC;
@@ -157,25 +161,43 @@ __global__ void __launch_bounds__(192, 1)
       fence_after();
 #pragma unroll 1
       for (int h = 0; h < MH; ++h) {
-        const int c = h * 128 + 32 * q + lane;                   // output channel of this lane
+        const int c0 = h * 128 + 32 * q;                         // first channel of this warp's block
+        if (c0 >= n_out) continue;                               // (warp-uniform) padding channels
+        const int c = c0 + lane;
         const float b = c < n_out ? __ldg(bias + c) : 0.f;
 #pragma unroll 1
         for (int r0 = 0; r0 < sp::BN; r0 += 32) {
           uint32_t r[32];
           tmem_ld32_nowait(tmem + ((uint32_t)(32 * q) << 16) + acc * Cfg::ACC_COLS + h * sp::BN + r0, r);
           tmem_wait_ld();
-          const int64_t row0 = tile * sp::BN + r0;
-          if (c < n_out) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              float v = __uint_as_float(r[j]) + b;
-              if (relu) v = fmaxf(v, 0.f);
-              if (row0 + j < M) {
-                if (c_f32) reinterpret_cast<float*>(C)[(row0 + j) * n_out + c] = v;
-                else reinterpret_cast<__nv_bfloat16*>(C)[(row0 + j) * n_out + c] = __float2bfloat16_rn(v);
+          for (int j = 0; j < 32; ++j) {                         // stage[row j][channel lane]
+            float v = __uint_as_float(r[j]) + b;
+            stg[j * 33 + lane] = relu ? fmaxf(v, 0.f) : v;
+          }
+          __syncwarp();
+          const int64_t row = tile * sp::BN + r0 + lane;         // lane = row now
+          if (row < M) {
+            const float* src = stg + lane * 33;
+            if (c_f32) {
+              float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(C) + row * n_out + c0);
+#pragma unroll
+              for (int u = 0; u < 8; ++u) dst[u] = make_float4(src[4 * u], src[4 * u + 1], src[4 * u + 2], src[4 * u + 3]);
+            } else {
+              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(C) + row * n_out + c0);
+#pragma unroll
+              for (int u = 0; u < 4; ++u) {
+                uint32_t p4[4];
+#pragma unroll
+                for (int t = 0; t < 4; ++t) {
+                  __nv_bfloat162 h2 = __floats2bfloat162_rn(src[8 * u + 2 * t], src[8 * u + 2 * t + 1]);
+                  p4[t] = *reinterpret_cast<uint32_t*>(&h2);
+                }
+                dst[u] = make_uint4(p4[0], p4[1], p4[2], p4[3]);
               }
             }
           }
+          __syncwarp();                                          // stage reused by the next block
         }
       }
       fence_before();
