@@ -17,7 +17,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpsim.so")
+LIB_PATH = os.environ.get("PSIM_LIB") or os.path.join(_HERE, "libpsim.so")   # PSIM_LIB: A/B experiments only
 
 OK, ERR_ARG, ERR_STATE, ERR_CUDA, ERR_NCCL, ERR_OOM, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 FP32, BF16 = 0, 1

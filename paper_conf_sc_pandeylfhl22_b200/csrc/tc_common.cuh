@@ -32,6 +32,22 @@ __device__ __forceinline__ bool mbar_try_wait(uint32_t a, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+// try_wait with a suspend-time hint: the thread sleeps until the phase completes (or the
+// hint, 10 ms, elapses) instead of spinning on issue slots its SM sub-partition's working
+// warps need
+__device__ __forceinline__ bool mbar_try_wait_sleep(uint32_t a, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2, %3;\n"
+      "selp.u32 %0, 1, 0, P1;\n"
+      "}\n"
+      : "=r"(ok)
+      : "r"(a), "r"(parity), "r"(0x989680u)
+      : "memory");
+  return ok != 0;
+}
 // Wait for the phase with this parity to complete.  Watchdog: a wait that has not
 // completed after ~2^36 clock cycles (~35 s) traps, so a pipeline bug surfaces as a
 // launch error instead of a hung GPU.
@@ -39,7 +55,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   if (mbar_try_wait(a, parity)) return;
   const long long t0 = clock64();
-  while (!mbar_try_wait(a, parity)) {
+  while (!mbar_try_wait_sleep(a, parity)) {
     if (clock64() - t0 > (1ll << 36)) __trap();
   }
 }
