@@ -229,41 +229,27 @@ __device__ __forceinline__ int update_subtrace_thread(const UpdateArgs& a, uint6
       goto done;
     }
   }
-  // Batches of 8 entries, double-buffered in registers: batch b + 2 is loaded while batch
-  // b + 1 is processed (the first batch was prefetched while the head ran), so at most every
-  // other batch waits on memory.  Loads only touch positions >= the next batch's start, which
-  // the in-place compaction (write index <= read index) has not reached yet.
-  QBatch bufA = first, bufB;
-  auto load_batch = [&](int e0, QBatch& B) {
-#pragma unroll
-    for (int t = 0; t < 8; ++t)
-      if (e0 + t < k) { const uint4 v = qb[(uint64_t)(e0 + t) * qn]; B.s[t] = v.x; B.f[t] = v.y; B.c[t] = v.z; B.w[t] = v.w; }
-  };
-  auto process = [&](const QBatch& B, int e0) {
+  for (int e0 = 0; e0 < n_in; e0 += 8) {
+    uint32_t vs[8], vf[8], vc[8], vw[8];
 #pragma unroll
     for (int t = 0; t < 8; ++t) {
       const int e = e0 + t;
-      if (e >= n_in) break;
-      uint32_t vs, vf, vc, vw;
-      if (e < k) { vs = B.s[t]; vf = B.f[t]; vc = B.c[t]; vw = B.w[t]; }
-      else { vs = push_s; vf = push_f; vc = push_c; vw = push_w; }   // e == k: the pushed entry
-      const int rem = (int)(vc & 0xFFFF) + (int)(vc >> 16) - (int)(clo - vf);   // retire - Clock
+      if (e < k) {
+        if (e0 == 0) { vs[t] = first.s[t]; vf[t] = first.f[t]; vc[t] = first.c[t]; vw[t] = first.w[t]; }   // prefetched
+        else { const uint4 v = qb[e * qn]; vs[t] = v.x; vf[t] = v.y; vc[t] = v.z; vw[t] = v.w; }
+      } else { vs[t] = push_s; vf[t] = push_f; vc[t] = push_c; vw[t] = push_w; }   // e == k: the pushed entry
+    }
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+      if (e0 + t >= n_in) break;
+      const int rem = (int)(vc[t] & 0xFFFF) + (int)(vc[t] >> 16) - (int)(clo - vf[t]);   // retire - Clock
       if (rem > 0) {
-        qb[(uint64_t)w * qn] = make_uint4(vs, vf, vc, vw);
+        qb[(uint64_t)w * qn] = make_uint4(vs[t], vf[t], vc[t], vw[t]);
         ++w;
         dmin = min(dmin, rem);
       } else {
-        nst += (int)(vw & 1u);
+        nst += (int)(vw[t] & 1u);
       }
-    }
-  };
-  if (8 < k) load_batch(8, bufB);
-  for (int e0 = 0; e0 < n_in; e0 += 16) {
-    process(bufA, e0);
-    if (e0 + 16 < k) load_batch(e0 + 16, bufA);
-    if (e0 + 8 < n_in) {
-      process(bufB, e0 + 8);
-      if (e0 + 24 < k) load_batch(e0 + 24, bufB);
     }
   }
   if (w > a.cap) {                                         // ROB-full stall: Clock = min retire (R5)
