@@ -597,14 +597,6 @@ struct HeadArgs {
   int force_predict;         // run the head even when teacher-forced
   long long* dbg;            // optional timestamps (PSIM_DEBUG_TIMING), slots 128..
   unsigned long long* ptile_sum;   // sum of P_tile over the tiles of the run (fc1 K statistics)
-  // N-split (few tiles: fewer tiles than half the SMs): CTA pair (2 t, 2 t + 1) shares tile t,
-  // CTA h computing fc1 outputs [128 h, 128 h + 128) and its part of fc2; half 1 hands its
-  // partial y to half 0 through ypart + ysync (release / acquire at gpu scope), half 0 runs
-  // the update.  Both CTAs of a pair are resident (grid = 2 x tiles <= SMs, 1 CTA per SM).
-  int nsplit;                // 1 or 2
-  float* ypart;              // [n][3] partial y of half 1
-  uint32_t* ysync;           // [ntiles] = stamp when tile t's partial y is written
-  uint32_t stamp;            // unique per launch
 };
 
 __global__ void __launch_bounds__(fh::THREADS, 1)
@@ -624,10 +616,6 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint64_t n = a.u.st.n;
   const uint32_t ntiles = (uint32_t)((n + fh::BM - 1) / fh::BM);
-  const int hs = (int)(blockIdx.x % (uint32_t)a.nsplit);          // N half of this CTA (0 if not split)
-  const uint32_t cta = blockIdx.x / (uint32_t)a.nsplit, ncta = gridDim.x / (uint32_t)a.nsplit;
-  const int bn = fh::BN / a.nsplit;                              // fc1 outputs of this CTA
-  const uint32_t stage_bytes = fh::A_BYTES + (uint32_t)bn * fh::BK * 2;
 
   uint64_t* cbar = tempty + 2;   // constant table + fc2 landed (bulk copies)
   uint64_t* yfull = cbar + 1;    // [2] epilogue -> update: y of a tile in sY[buf]
@@ -660,12 +648,12 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   grid_dep_launch_dependents();
   const bool run_head = (a.u.forced == nullptr) || a.force_predict;
   int npre = 0;   // producer: k-blocks of the first tile whose B half was issued before the wait
-  if (warp == 0 && lane == 0 && run_head && cta < ntiles) {
-    npre = min(2 * (int)a.tileP[cta], fh::STAGES);
+  if (warp == 0 && lane == 0 && run_head && blockIdx.x < ntiles) {
+    npre = min(2 * (int)a.tileP[blockIdx.x], fh::STAGES);
     for (int kb = 0; kb < npre; ++kb) {
       uint8_t* sa = sm + kb * fh::STAGE;
-      mbar_expect_tx(full + kb, stage_bytes);
-      tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, hs * 128, l2_policy_evict_last());
+      mbar_expect_tx(full + kb, fh::STAGE);
+      tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0, l2_policy_evict_last());
     }
   }
   grid_dep_wait();
@@ -677,7 +665,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const uint64_t polA = l2_policy_evict_first(), polB = l2_policy_evict_last();
       uint32_t stage = 0, phase = 0;
       uint32_t it = 0;
-      for (uint32_t tt = cta; tt < ntiles; tt += ncta, ++it) {
+      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
         const int nk = 2 * a.tileP[tt];
         PSIM_TS(128);
         for (int kb = 0; kb < nk; ++kb) {
@@ -686,9 +674,9 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
             tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
           } else {
             mbar_wait(empty + stage, phase ^ 1);
-            mbar_expect_tx(full + stage, stage_bytes);
+            mbar_expect_tx(full + stage, fh::STAGE);
             tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
-            tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, hs * 128, polB);
+            tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0, polB);
           }
           if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
         }
@@ -697,9 +685,9 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     }
   } else if (warp == 1) {
     if (lane == 0 && run_head) {   // ---- MMA issuer
-      const uint32_t idesc = idesc_bf16(fh::BM, bn);
+      constexpr uint32_t idesc = idesc_bf16(fh::BM, fh::BN);
       uint32_t stage = 0, phase = 0, it = 0;
-      for (uint32_t tt = cta; tt < ntiles; tt += ncta, ++it) {
+      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
         const int nk = 2 * a.tileP[tt];
         const int acc = it & 1;
         PSIM_TS(132);
@@ -725,7 +713,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     const int m = q * 32 + lane;
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t it = 0;
-    for (uint32_t tt = cta; tt < ntiles; tt += ncta, ++it) {
+    for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
       const int acc = it & 1, yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const int ptile = a.tileP[tt];
@@ -737,9 +725,8 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         wait_full(tfull + acc, it >> 1);
         if (q == 2) PSIM_TS(141);
         fence_after();
-        if (hs == 0) { y0 = sW2[768]; y1 = sW2[769]; y2 = sW2[770]; }   // fc2 bias once per row
-        const float* Trow = sT + pb * fh::T_STRIDE + hs * 128;           // this CTA's fc1 outputs
-        const float* w2b = sW2 + hs * 128;
+        y0 = sW2[768]; y1 = sW2[769]; y2 = sW2[770];
+        const float* Trow = sT + pb * fh::T_STRIDE;
         // fc1 = F (positions < P_tile; rows [P_b, P_tile) are zero) + T[P_b]; ReLU; fc2 (R16, R18).
         // Two TMEM loads in flight (the next 32 columns load while these are consumed) and
         // two partial sums per output (halves the dependent FMA chains).
@@ -752,9 +739,9 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
           for (int j4 = 0; j4 < 8; ++j4) {
             const int col = cc * 32 + j4 * 4;
             const float4 tv = *reinterpret_cast<const float4*>(Trow + col);
-            const float4 w0 = *reinterpret_cast<const float4*>(w2b + col);
-            const float4 w1 = *reinterpret_cast<const float4*>(w2b + 256 + col);
-            const float4 w2v = *reinterpret_cast<const float4*>(w2b + 512 + col);
+            const float4 w0 = *reinterpret_cast<const float4*>(sW2 + col);
+            const float4 w1 = *reinterpret_cast<const float4*>(sW2 + 256 + col);
+            const float4 w2v = *reinterpret_cast<const float4*>(sW2 + 512 + col);
             const float f0 = ptile > 0 ? __uint_as_float(r0[j4 * 4]) : 0.f, f1 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 1]) : 0.f;
             const float f2 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 2]) : 0.f, f3 = ptile > 0 ? __uint_as_float(r0[j4 * 4 + 3]) : 0.f;
             const float h0 = fmaxf(f0 + tv.x, 0.f), h1 = fmaxf(f1 + tv.y, 0.f);
@@ -765,41 +752,18 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
           }
         };
 #pragma unroll 1
-        for (int cc = 0; cc < bn / 32; cc += 2) {
+        for (int cc = 0; cc < fh::BN / 32; cc += 2) {
           tmem_wait_ld();                                   // columns cc (ra) landed
           tmem_ld32_nowait(tbase + (cc + 1) * 32, rb);
           consume(ra, cc);
           tmem_wait_ld();                                   // columns cc + 1 (rb) landed
-          if (cc + 2 < bn / 32) tmem_ld32_nowait(tbase + (cc + 2) * 32, ra);
+          if (cc + 2 < fh::BN / 32) tmem_ld32_nowait(tbase + (cc + 2) * 32, ra);
           consume(rb, cc + 1);
         }
         y0 += z0; y1 += z1; y2 += z2;
         fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(tempty + acc);
-      }
-      if (a.nsplit == 2) {   // N-split: half 1 publishes its partial y, half 0 adds it
-        if (hs == 1) {
-          if (run_head) {
-            if (b < n) { a.ypart[b * 3] = y0; a.ypart[b * 3 + 1] = y1; a.ypart[b * 3 + 2] = y2; }
-            __threadfence();
-            named_bar_sync(4, 128);
-            if (m == 0) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a.ysync + tt), "r"(a.stamp) : "memory");
-          }
-          continue;                                     // half 1 has no update
-        }
-        if (run_head) {
-          if (m == 0) {
-            const long long t0 = clock64();
-            uint32_t v;
-            do {
-              asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(a.ysync + tt) : "memory");
-              if (clock64() - t0 > (1ll << 36)) __trap();   // watchdog (the partner CTA is resident)
-            } while (v != a.stamp);
-          }
-          named_bar_sync(4, 128);
-          if (b < n) { y0 += __ldcg(a.ypart + b * 3); y1 += __ldcg(a.ypart + b * 3 + 1); y2 += __ldcg(a.ypart + b * 3 + 2); }
-        }
       }
       wait_empty(yempty + yb, it >> 1);
       float* yrow = sY + (yb * 128 + m) * 3;
@@ -808,13 +772,13 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       if (lane == 0) mbar_arrive(yfull + yb);
       if (q == 2) PSIM_TS(142);
     }
-  } else if (hs == 0) {   // ---- update (group 0: warps 6..9 even tiles, group 1: 10..13 odd tiles), thread per sub-trace
+  } else {   // ---- update (group 0: warps 6..9 even tiles, group 1: 10..13 odd tiles), thread per sub-trace
     const int grp = (warp - 6) >> 2;
     const int q = (warp - 6) & 3;
     const int m = q * 32 + lane;
     int* sPg = sP + grp * 16;
     uint32_t it = grp;
-    for (uint32_t tt = cta + grp * ncta; tt < ntiles; tt += 2 * ncta, it += 2) {
+    for (uint32_t tt = blockIdx.x + grp * gridDim.x; tt < ntiles; tt += 2 * gridDim.x, it += 2) {
       const int yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const bool inb = b < n;
@@ -1173,15 +1137,8 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
   a.dbg = debug_buffer(step);
   a.ptile_sum = u.st.ptile_sum;
   const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
-  // N-split when at most half the SMs would be busy (G >= 4 slices): two CTAs per tile
-  // (PSIM_FC1_SPLIT=0 disables); every CTA is then resident (grid <= SMs, 1 CTA per SM)
-  static const bool allow_split = [] { const char* e = getenv("PSIM_FC1_SPLIT"); return !(e && atoi(e) == 0); }();
-  a.nsplit = (allow_split && f.ypart && 2 * ntiles <= (uint64_t)sm_count()) ? 2 : 1;
-  a.ypart = f.ypart;
-  a.ysync = f.ysync;
-  a.stamp = ++f.launch_stamp;
-  const int grid = a.nsplit == 2 ? (int)(2 * ntiles) : (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
-  launch_pdl(fc1_head_kernel, grid, fh::THREADS, fh::SMEM, st, f.mapA, a.nsplit == 2 ? f.mapB128 : f.mapB, a);
+  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
+  launch_pdl(fc1_head_kernel, grid, fh::THREADS, fh::SMEM, st, f.mapA, f.mapB, a);
 }
 
 bool fused_make_weight_maps(FusedC3& f) {
@@ -1204,8 +1161,7 @@ bool fused_make_trace_map(FusedC3& f, uint64_t rows) {
 }
 
 bool fused_make_maps(FusedC3& f, uint64_t n) {
-  return map2d(&f.mapA, f.a4, n, 14 * 128, fh::BM) && map2d(&f.mapB, f.wfc1, 256, 14 * 128, fh::BN) &&
-         map2d(&f.mapB128, f.wfc1, 256, 14 * 128, fh::BN / 2);
+  return map2d(&f.mapA, f.a4, n, 14 * 128, fh::BM) && map2d(&f.mapB, f.wfc1, 256, 14 * 128, fh::BN);
 }
 
 }  // namespace psim

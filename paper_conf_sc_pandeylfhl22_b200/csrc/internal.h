@@ -215,10 +215,6 @@ struct FusedC3 {
   uint8_t* tileP[2] = {nullptr, nullptr};   // [ceil(n/128)] P_tile by step parity
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
   CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
-  CUtensorMap mapB128;                // wfc1 with a 128-row box (fc1_head N-split)
-  float* ypart = nullptr;             // [n][3] partial y of the N-split's second CTA (owned)
-  uint32_t* ysync = nullptr;          // [ceil(n/128)] per-tile hand-off stamps (owned)
-  uint32_t launch_stamp = 0;          // fc1_head launches so far (hand-off stamps)
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
   CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][48] (box 48 x 1, SWIZZLE_128B)
   uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)

@@ -276,8 +276,6 @@ void psim_destroy(psim_ctx* ctx) {
   dfree(ctx->fused.tileP[0]);
   dfree(ctx->fused.tileP[1]);
   dfree(ctx->fused.a4);
-  dfree(ctx->fused.ypart);
-  dfree(ctx->fused.ysync);
   for (Cohort& c : ctx->cohorts) {
     dfree(c.blocks); dfree(c.count); dfree(c.tileP[0]); dfree(c.tileP[1]);
     if (c.st) cudaStreamDestroy(c.st);
@@ -758,9 +756,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     const uint64_t nn = std::max<uint64_t>(n, 1);
     if (fz.cap_n != nn) {
       dfree(fz.blocks); dfree(fz.count); dfree(fz.tileP[0]); dfree(fz.tileP[1]); dfree(fz.a4);
-      dfree(fz.ypart); dfree(fz.ysync);
       fz.blocks = nullptr; fz.count = nullptr; fz.tileP[0] = fz.tileP[1] = nullptr; fz.a4 = nullptr;
-      fz.ypart = nullptr; fz.ysync = nullptr;
       const uint64_t nt = (nn + 127) / 128;
       CK(cudaMalloc(&fz.blocks, nn * 14 * 16));
       CK(cudaMalloc(&fz.count, 16));
@@ -768,10 +764,6 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       CK(cudaMalloc(&fz.tileP[1], nt + 16));
       CK(cudaMalloc(&fz.a4, nn * 14 * 128 * 2));
       CK(cudaMemset(fz.a4, 0, nn * 14 * 128 * 2));
-      CK(cudaMalloc(&fz.ypart, nn * 12 + 16));
-      CK(cudaMalloc(&fz.ysync, nt * 4 + 16));
-      CK(cudaMemset(fz.ysync, 0, nt * 4 + 16));
-      fz.launch_stamp = 0;
       if (!fused_make_maps(fz, nn)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for the fused path");
       fz.cap_n = nn;
     }
