@@ -1030,7 +1030,7 @@ static bool map2d(CUtensorMap* m, const void* ptr, uint64_t rows, uint64_t cols,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-static int sm_count() {
+int sm_count() {
   static int n = 0;
   if (!n) {
     int dev = 0;
@@ -1113,7 +1113,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   // the block count is only known on the device: launch one persistent CTA per SM
   // (n*14 blocks at most); CTAs with no tile exit after setup.
   const uint64_t max_tiles = (n * 14 + cs::TILE - 1) / cs::TILE;
-  const int grid = (int)std::min<uint64_t>(max_tiles, (uint64_t)sm_count());
+  const int grid = (int)std::min<uint64_t>(max_tiles, (uint64_t)(f.grid_cap > 0 ? f.grid_cap : sm_count()));
   launch_pdl(conv_stack_kernel, grid, cs::THREADS, cs::SMEM, st, a, f.mapW1, f.mapW2, f.mapW3, f.mapX);
 }
 
@@ -1137,7 +1137,7 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
   a.dbg = debug_buffer(step);
   a.ptile_sum = u.st.ptile_sum;
   const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
-  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)sm_count());
+  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)(f.grid_cap > 0 ? f.grid_cap : sm_count()));
   launch_pdl(fc1_head_kernel, grid, fh::THREADS, fh::SMEM, st, f.mapA, f.mapB, a);
 }
 

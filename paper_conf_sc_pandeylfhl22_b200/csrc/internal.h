@@ -215,6 +215,8 @@ struct FusedC3 {
   uint8_t* tileP[2] = {nullptr, nullptr};   // [ceil(n/128)] P_tile by step parity
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
   CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
+  int grid_cap = 0;                   // max CTAs of the persistent fused kernels (0: one per SM);
+                                      // cohorts with disjoint SM shares run side by side
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
   CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][48] (box 48 x 1, SWIZZLE_128B)
   uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)
@@ -235,6 +237,7 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
                      cudaStream_t st);
 bool fused_make_maps(FusedC3& f, uint64_t n);
+int sm_count();   // SMs of the current device
 bool fused_make_weight_maps(FusedC3& f);
 // gather4 map of f.trace16 with rows + 1 rows (the last one zero); sets f.zero_row
 bool fused_make_trace_map(FusedC3& f, uint64_t rows);

@@ -938,6 +938,10 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
       ch.fz = ctx->fused;
       ch.fz.blocks = ch.blocks; ch.fz.count = ch.count; ch.fz.tileP[0] = ch.tileP[0]; ch.fz.tileP[1] = ch.tileP[1];
       ch.fz.a4 = ctx->fused.a4 + b0 * 14 * 128;
+      // PSIM_COHORT_SMS=1: each cohort's persistent kernels get a disjoint share of the SMs,
+      // so one cohort's conv_stack runs beside another's fc1_head instead of queueing behind it
+      static const bool share = [] { const char* e = getenv("PSIM_COHORT_SMS"); return e && atoi(e) != 0; }();
+      ch.fz.grid_cap = share ? std::max(1, sm_count() / ncoh) : 0;
       if (!fused_make_maps(ch.fz, ch.n)) FAIL(PSIM_ERR_CUDA, "cuTensorMapEncodeTiled failed for a cohort");
       CK(cudaStreamWaitEvent(ch.st, ctx->ev[3], 0));
       launch_fused_init(ch.fz, ctx->st.ws + ch.b0, ch.n, ch.st);

@@ -1,0 +1,6 @@
+# cohorts with disjoint SM shares (PSIM_COHORTS, PSIM_COHORT_SMS) at the G = 8 / 4 / 1 slices
+for g in 8 4 1; do for cfg in "1 0" "2 0" "2 1" "3 1" "4 1"; do set -- $cfg
+  emu=""; [ $g -gt 1 ] && emu="--emulate-rank 0/$g"
+  PSIM_COHORTS=$1 PSIM_COHORT_SMS=$2 timeout 300 python bench.py --steps 3 --warmup 2 --no-cpu --no-e2e $emu 2>/dev/null | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print('G=$g cohorts=$1 sms=$2 VALUE', round(d['value'],1), 'ms', round(d['ms_per_step'],1), 'cycles', d['total_cycles'])"
+done; done
