@@ -258,8 +258,6 @@ __device__ __forceinline__ void bias_relu_pack32(const uint32_t (&r)[32], const 
     out[2 * c + 1] = pack_bf16_relu(__uint_as_float(r[4 * c + 2]) + bv.z, __uint_as_float(r[4 * c + 3]) + bv.w);
   }
 }
-// 16-byte store into a K-major SWIZZLE_128B tile: row m (128 B), logical
-// 16-byte chunk c (0..7) lands in physical chunk c ^ (m & 7).
 // one elected lane of a converged warp (the MMA / TMA issue idiom: the whole warp runs
 // the issue loop so its operands stay warp-uniform, one lane issues)
 __device__ __forceinline__ bool elect_one() {
@@ -272,6 +270,8 @@ template <int N>
 __device__ __forceinline__ void setmaxnreg_dec() { asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N)); }
 template <int N>
 __device__ __forceinline__ void setmaxnreg_inc() { asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N)); }
+// 16-byte store into a K-major SWIZZLE_128B tile: row m (128 B), logical
+// 16-byte chunk c (0..7) lands in physical chunk c ^ (m & 7).
 __device__ __forceinline__ void st_sw128(uint8_t* atom, int m, int c, uint4 v) {
   *reinterpret_cast<uint4*>(atom + m * 128 + ((c ^ (m & 7)) << 4)) = v;
 }
