@@ -71,6 +71,11 @@ extern "C" {
                                 tcgen05.mma.sp GEMM of the layer-wise path.  load_model returns ARG
                                 if a group holds more than 2 nonzeros, UNSUPPORTED for other
                                 architectures or fp32                                          */
+#define PSIM_FC1_PAIR 32u    /* fused C3 path: fc1_head on 2-SM MMAs (tcgen05.mma.cta_group::2,
+                                M = 256 over a cluster of two CTAs, each staging its own tile's
+                                activations and half of the fc1 weights; multicast commits,
+                                2-SM TMA).  Same results; measured slower on B200 (fc1_head is
+                                not bound by its weight stream), so off by default       */
 #define PSIM_PROFILE 2u      /* time kernel classes with CUDA events on the launch stream: every
                                 launch outside the step loop and the launches of every 16th
                                 lockstep step (events between all launches would serialise the

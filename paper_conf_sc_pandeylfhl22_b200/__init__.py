@@ -27,6 +27,7 @@ PROFILE = 2
 FORCE_PREDICT = 4
 LAYERWISE = 8
 SPARSE24 = 16
+FC1_PAIR = 32
 MAX_CAP = 110
 MAX_INTERVAL = 262144   # PSIM_MAX_INTERVAL
 NATTR = 47
@@ -173,7 +174,7 @@ class Simulator:
                  rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
                  stream=None, record_rows: bool = False, chunk_steps: int = 0, profile: bool = False,
                  force_predict: bool = False, layerwise: bool = False, correction_limit: int = 0,
-                 interval: int = 0, sparse24: bool = False):
+                 interval: int = 0, sparse24: bool = False, fc1_pair: bool = False):
         self._keep = []
         idbuf = None
         if nccl_id is not None:
@@ -186,7 +187,7 @@ class Simulator:
                   stream=ctypes.c_void_p(int(stream)) if stream is not None else None,
                   flags=(RECORD_ROWS if record_rows else 0) | (PROFILE if profile else 0)
                   | (FORCE_PREDICT if force_predict else 0) | (LAYERWISE if layerwise else 0)
-                  | (SPARSE24 if sparse24 else 0),
+                  | (SPARSE24 if sparse24 else 0) | (FC1_PAIR if fc1_pair else 0),
                   correction_limit=correction_limit, interval=interval)
         h = ctypes.c_void_p()
         rc = lib().psim_create(ctypes.byref(o), ctypes.byref(h))

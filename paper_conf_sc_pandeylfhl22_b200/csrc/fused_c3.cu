@@ -575,7 +575,12 @@ constexpr int Y_OFF = W2_OFF + (3 * 256 + 4) * 4;   // float [128][3]
 constexpr int P_OFF = Y_OFF + 2 * 128 * 3 * 4;      // int [2][16] tile scan scratch per update group
 constexpr int H_OFF = P_OFF + 32 * 4;               // uint [112] k histogram of this CTA
 constexpr int BAR_OFF = (H_OFF + 112 * 4 + 7) & ~7;
-constexpr int SMEM = BAR_OFF + 160 + 1024;
+constexpr int SMEM = BAR_OFF + 256 + 1024;
+// pair mode (fc1 on 2-SM MMAs): a cluster of two CTAs computes two tiles with one
+// tcgen05.mma.cta_group::2 (M = 256): each CTA stages its own tile's a4 rows and HALF of the
+// W_fc1 slice (N rows 128 r .. 128 r + 127), so the W_fc1 stream per SM halves; smaller
+// stages (32 KB) -> 6 of them in the same 192 KB
+constexpr int PSTAGE = A_BYTES + B_BYTES / 2, PSTAGES = (STAGES * STAGE) / PSTAGE;
 constexpr int THREADS = 448;   // warp 0 TMA, 1 MMA, 2-5 epilogue (F -> y), 6-9 / 10-13 update groups (even / odd tiles)
 }  // namespace fh
 
@@ -599,8 +604,11 @@ struct HeadArgs {
   unsigned long long* ptile_sum;   // sum of P_tile over the tiles of the run (fc1 K statistics)
 };
 
+template <bool kPair>
 __global__ void __launch_bounds__(fh::THREADS, 1)
     fc1_head_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, HeadArgs a) {
+  constexpr int kStages = kPair ? fh::PSTAGES : fh::STAGES;
+  constexpr int kStage = kPair ? fh::PSTAGE : fh::STAGE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   float* sT = reinterpret_cast<float*>(sm + fh::T_OFF);
@@ -608,14 +616,25 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   int* sP = reinterpret_cast<int*>(sm + fh::P_OFF);
   unsigned int* sHist = reinterpret_cast<unsigned int*>(sm + fh::H_OFF);
   uint64_t* full = reinterpret_cast<uint64_t*>(sm + fh::BAR_OFF);
-  uint64_t* empty = full + fh::STAGES;
-  uint64_t* tfull = empty + fh::STAGES;
+  uint64_t* empty = full + kStages;
+  uint64_t* tfull = empty + kStages;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = nullptr;
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint64_t n = a.u.st.n;
   const uint32_t ntiles = (uint32_t)((n + fh::BM - 1) / fh::BM);
+  // tile schedule: single mode, CTA c takes tiles c, c + G, ...; pair mode, the CTA of rank r in
+  // cluster q takes tiles 2 (q + k Q) + r (k = 0, 1, ...; a tile >= ntiles is empty: its a4 rows
+  // read as zero past the tensor, its rows are skipped by the epilogue and the update)
+  const uint32_t rank = kPair ? cluster_ctarank() : 0u;
+  const uint32_t t0 = kPair ? 2 * cluster_id_x() + rank : blockIdx.x;
+  const uint32_t tstep = kPair ? 2 * ncluster_x() : gridDim.x;
+  const uint32_t tend = kPair ? ((ntiles + 1) & ~1u) : ntiles;   // pairs cover the odd last tile
+  auto tileP_of = [&](uint32_t t) -> int { return t < ntiles ? (int)a.tileP[t] : 0; };
+  auto nk_of = [&](uint32_t t) -> int {                           // k-blocks of tile t (pair: of its pair)
+    return kPair ? 2 * max(tileP_of(t & ~1u), tileP_of(t | 1u)) : 2 * tileP_of(t);
+  };
 
   uint64_t* cbar = tempty + 2;   // constant table + fc2 landed (bulk copies)
   uint64_t* yfull = cbar + 1;    // [2] epilogue -> update: y of a tile in sY[buf]
@@ -625,8 +644,9 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   if (tid < 3) sW2[768 + tid] = a.b2[tid];
   for (int idx = tid; idx < 112; idx += fh::THREADS) sHist[idx] = 0;
   if (tid == 0) {
-    for (int s = 0; s < fh::STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(tfull + i, 1); mbar_init(tempty + i, 4); }
+    for (int s = 0; s < kStages; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    // pair mode: tempty of the even CTA collects the epilogue warps of both CTAs
+    for (int i = 0; i < 2; ++i) { mbar_init(tfull + i, 1); mbar_init(tempty + i, kPair ? 8 : 4); }
     mbar_init(cbar, 1);
     for (int i = 0; i < 2; ++i) { mbar_init(yfull + i, 4); mbar_init(yempty + i, 4); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -634,9 +654,13 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     for (int r = 0; r < 15; ++r) bulk_g2s(sT + r * fh::T_STRIDE, a.T + r * 256, 1024, cbar);
     bulk_g2s(sW2, a.w2, 3 * 1024, cbar);
   }
-  if (warp == 1) tmem_alloc(tmem_slot, 512);
+  if (warp == 1) {
+    if constexpr (kPair) tmem_alloc_2sm(tmem_slot, 512);   // both CTAs, same warp
+    else tmem_alloc(tmem_slot, 512);
+  }
   fence_before();
   __syncthreads();
+  if constexpr (kPair) cluster_sync();   // barrier inits visible to the peer before any remote use
   fence_after();
   const uint32_t tmem = *tmem_slot;
   // PDL: every role waits (griddepcontrol.wait) for a4, block counts and queue state of
@@ -648,12 +672,17 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   grid_dep_launch_dependents();
   const bool run_head = (a.u.forced == nullptr) || a.force_predict;
   int npre = 0;   // producer: k-blocks of the first tile whose B half was issued before the wait
-  if (warp == 0 && lane == 0 && run_head && blockIdx.x < ntiles) {
-    npre = min(2 * (int)a.tileP[blockIdx.x], fh::STAGES);
+  if (warp == 0 && lane == 0 && run_head && t0 < tend) {
+    npre = min(nk_of(t0), kStages);
     for (int kb = 0; kb < npre; ++kb) {
-      uint8_t* sa = sm + kb * fh::STAGE;
-      mbar_expect_tx(full + kb, fh::STAGE);
-      tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0, l2_policy_evict_last());
+      uint8_t* sa = sm + kb * kStage;
+      if constexpr (kPair) {
+        if (rank == 0) mbar_expect_tx(full + kb, 2 * kStage);   // both CTAs' A + B-half bytes
+        tma_load_2d_2sm(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 128 * (int)rank, l2_policy_evict_last());
+      } else {
+        mbar_expect_tx(full + kb, fh::STAGE);
+        tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + kb, kb * fh::BK, 0, l2_policy_evict_last());
+      }
     }
   }
   grid_dep_wait();
@@ -665,12 +694,19 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       const uint64_t polA = l2_policy_evict_first(), polB = l2_policy_evict_last();
       uint32_t stage = 0, phase = 0;
       uint32_t it = 0;
-      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
-        const int nk = 2 * a.tileP[tt];
+      for (uint32_t tt = t0; tt < tend; tt += tstep, ++it) {
+        const int nk = nk_of(tt);
         PSIM_TS(128);
         for (int kb = 0; kb < nk; ++kb) {
-          uint8_t* sa = sm + stage * fh::STAGE;
-          if (it == 0 && kb < npre) {                 // B already in flight (issued before the PDL wait)
+          uint8_t* sa = sm + stage * kStage;
+          if constexpr (kPair) {
+            if (!(it == 0 && kb < npre)) {              // else B already in flight (issued before the PDL wait)
+              mbar_wait(empty + stage, phase ^ 1);      // released by the pair's MMA commit (multicast)
+              if (rank == 0) mbar_expect_tx(full + stage, 2 * kStage);
+              tma_load_2d_2sm(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 128 * (int)rank, polB);
+            }
+            tma_load_2d_2sm(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
+          } else if (it == 0 && kb < npre) {            // B already in flight (issued before the PDL wait)
             tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
           } else {
             mbar_wait(empty + stage, phase ^ 1);
@@ -678,17 +714,17 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
             tma_load_2d_hint(sa, &tmA, full + stage, kb * fh::BK, (int)(tt * fh::BM), polA);
             tma_load_2d_hint(sa + fh::A_BYTES, &tmB, full + stage, kb * fh::BK, 0, polB);
           }
-          if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
+          if (++stage == kStages) { stage = 0; phase ^= 1; }
         }
         PSIM_TS(129);
       }
     }
   } else if (warp == 1) {
-    if (lane == 0 && run_head) {   // ---- MMA issuer
-      constexpr uint32_t idesc = idesc_bf16(fh::BM, fh::BN);
+    if (lane == 0 && run_head && rank == 0) {   // ---- MMA issuer (pair mode: the even CTA issues for both)
+      constexpr uint32_t idesc = idesc_bf16(kPair ? 2 * fh::BM : fh::BM, fh::BN);
       uint32_t stage = 0, phase = 0, it = 0;
-      for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
-        const int nk = 2 * a.tileP[tt];
+      for (uint32_t tt = t0; tt < tend; tt += tstep, ++it) {
+        const int nk = nk_of(tt);
         const int acc = it & 1;
         PSIM_TS(132);
         wait_empty(tempty + acc, it >> 1);
@@ -697,14 +733,21 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         for (int kb = 0; kb < nk; ++kb) {
           mbar_wait(full + stage, phase);
           fence_after();
-          const uint32_t sa = smem_u32(sm + stage * fh::STAGE), sb = sa + fh::A_BYTES;
+          const uint32_t sa = smem_u32(sm + stage * kStage), sb = sa + fh::A_BYTES;
 #pragma unroll
-          for (int k = 0; k < fh::BK / 16; ++k)
-            mma_bf16(tmem + acc * fh::BN, sw128_desc(sa + 32 * k), sw128_desc(sb + 32 * k), idesc, (kb | k) != 0);
-          mma_commit(empty + stage);
-          if (++stage == fh::STAGES) { stage = 0; phase ^= 1; }
+          for (int k = 0; k < fh::BK / 16; ++k) {
+            if constexpr (kPair)   // A: 128 rows per CTA (M = 256), B: 128 N-rows per CTA (N = 256)
+              mma_bf16_2sm(tmem + acc * fh::BN, sw128_desc(sa + 32 * k), sw128_desc(sb + 32 * k), idesc, (kb | k) != 0);
+            else
+              mma_bf16(tmem + acc * fh::BN, sw128_desc(sa + 32 * k), sw128_desc(sb + 32 * k), idesc, (kb | k) != 0);
+          }
+          if constexpr (kPair) mma_commit_2sm_mc(empty + stage, 0x3);   // frees the stage in both CTAs
+          else mma_commit(empty + stage);
+          if (++stage == kStages) { stage = 0; phase ^= 1; }
         }
-        mma_commit(tfull + acc);   // nk == 0: arrives once the earlier MMAs are done
+        // accumulator ready (nk == 0: arrives once the earlier MMAs are done)
+        if constexpr (kPair) mma_commit_2sm_mc(tfull + acc, 0x3);
+        else mma_commit(tfull + acc);
         PSIM_TS(134);
       }
     }
@@ -713,10 +756,10 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     const int m = q * 32 + lane;
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t it = 0;
-    for (uint32_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x, ++it) {
+    for (uint32_t tt = t0; tt < tend; tt += tstep, ++it) {
       const int acc = it & 1, yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
-      const int ptile = a.tileP[tt];
+      const int ptile = tileP_of(tt);
       const int kb = b < n ? a.u.st.count[b] : 0;   // read before this tile's update (y handoff orders it)
       const int pb = min((kb + 8) >> 3, 14);        // computed positions of this sub-trace
       float y0 = 0.f, y1 = 0.f, y2 = 0.f;
@@ -763,7 +806,10 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         y0 += z0; y1 += z1; y2 += z2;
         fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(tempty + acc);
+        if (lane == 0) {
+          if constexpr (kPair) mbar_arrive_cluster(mapa_shared(tempty + acc, 0));   // the issuing CTA's barrier
+          else mbar_arrive(tempty + acc);
+        }
       }
       wait_empty(yempty + yb, it >> 1);
       float* yrow = sY + (yb * 128 + m) * 3;
@@ -778,12 +824,12 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     const int m = q * 32 + lane;
     int* sPg = sP + grp * 16;
     uint32_t it = grp;
-    for (uint32_t tt = blockIdx.x + grp * gridDim.x; tt < ntiles; tt += 2 * gridDim.x, it += 2) {
+    for (uint32_t tt = t0 + grp * tstep; tt < tend; tt += 2 * tstep, it += 2) {
       const int yb = it & 1;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const bool inb = b < n;
       if (q == 0) PSIM_TS(145);
-      const int tileP_cur = a.tileP[tt];
+      const int tileP_cur = tileP_of(tt);
       int64_t ws = 0, s_b = 0, nsteps = 0, clock = 0;
       int kb = 0;
       uint32_t rmin = 0;
@@ -836,7 +882,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
         const int total = sPg[0] + sPg[1] + sPg[2] + sPg[3];
         sPg[8] = total ? (int)atomicAdd(a.next_count, (uint32_t)total) : 0;
         const int ptn = max(max(sPg[4], sPg[5]), max(sPg[6], sPg[7]));
-        a.tileP_next[tt] = (uint8_t)ptn;
+        if (tt < ntiles) a.tileP_next[tt] = (uint8_t)ptn;
         if (a.ptile_sum && tileP_cur > 0) atomicAdd(a.ptile_sum, (unsigned long long)tileP_cur);
       }
       named_bar_sync(2 + grp, 128);
@@ -852,9 +898,11 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     if (sHist[k]) atomicAdd(a.u.st.k_hist + k, (unsigned long long)sHist[k]);
   fence_before();
   __syncthreads();
+  if constexpr (kPair) cluster_sync();   // the peer no longer signals this CTA's barriers
   if (warp == 1) {
     fence_after();
-    tmem_dealloc(tmem, 512);
+    if constexpr (kPair) tmem_dealloc_2sm(tmem, 512);
+    else tmem_dealloc(tmem, 512);
   }
 }
 
@@ -1120,8 +1168,24 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
 void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t step, bool force_predict,
                      cudaStream_t st) {
   static bool attr = false;
+  static int max_pairs = 0;
   if (!attr) {
-    cudaFuncSetAttribute(fc1_head_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, fh::SMEM);
+    cudaFuncSetAttribute(fc1_head_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, fh::SMEM);
+    cudaFuncSetAttribute(fc1_head_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, fh::SMEM);
+    // co-resident 2-CTA clusters of the pair kernel (SM pairs within a GPC)
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * (unsigned)sm_count());
+    cfg.blockDim = dim3(fh::THREADS);
+    cfg.dynamicSmemBytes = fh::SMEM;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    if (cudaOccupancyMaxActiveClusters(&max_pairs, fc1_head_kernel<true>, &cfg) != cudaSuccess) {
+      max_pairs = 0;
+      cudaGetLastError();
+    }
     attr = true;
   }
   HeadArgs a;
@@ -1137,8 +1201,28 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
   a.dbg = debug_buffer(step);
   a.ptile_sum = u.st.ptile_sum;
   const uint64_t ntiles = (u.st.n + fh::BM - 1) / fh::BM;
-  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)(f.grid_cap > 0 ? f.grid_cap : sm_count()));
-  launch_pdl(fc1_head_kernel, grid, fh::THREADS, fh::SMEM, st, f.mapA, f.mapB, a);
+  const int cap = f.grid_cap > 0 ? f.grid_cap : sm_count();
+  // pair mode (psim_opts flag PSIM_FC1_PAIR): fc1 on 2-SM MMAs, two tiles per CTA pair
+  if (f.pair && max_pairs > 0 && ntiles >= 2) {
+    const uint64_t pairs = std::min<uint64_t>(std::min<uint64_t>((ntiles + 1) / 2, (uint64_t)max_pairs),
+                                              (uint64_t)std::max(1, cap / 2));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(2 * pairs));
+    cfg.blockDim = dim3(fh::THREADS);
+    cfg.dynamicSmemBytes = fh::SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    at[1].id = cudaLaunchAttributeClusterDimension;
+    at[1].val.clusterDim.x = 2; at[1].val.clusterDim.y = 1; at[1].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 2;
+    cudaLaunchKernelEx(&cfg, fc1_head_kernel<true>, f.mapA, f.mapB128, a);
+    return;
+  }
+  const int grid = (int)std::min<uint64_t>(ntiles, (uint64_t)cap);
+  launch_pdl(fc1_head_kernel<false>, grid, fh::THREADS, fh::SMEM, st, f.mapA, f.mapB, a);
 }
 
 bool fused_make_weight_maps(FusedC3& f) {
@@ -1161,7 +1245,8 @@ bool fused_make_trace_map(FusedC3& f, uint64_t rows) {
 }
 
 bool fused_make_maps(FusedC3& f, uint64_t n) {
-  return map2d(&f.mapA, f.a4, n, 14 * 128, fh::BM) && map2d(&f.mapB, f.wfc1, 256, 14 * 128, fh::BN);
+  return map2d(&f.mapA, f.a4, n, 14 * 128, fh::BM) && map2d(&f.mapB, f.wfc1, 256, 14 * 128, fh::BN) &&
+         map2d(&f.mapB128, f.wfc1, 256, 14 * 128, fh::BN / 2);   // pair mode: each CTA's 128 N-rows
 }
 
 }  // namespace psim

@@ -215,6 +215,8 @@ struct FusedC3 {
   uint8_t* tileP[2] = {nullptr, nullptr};   // [ceil(n/128)] P_tile by step parity
   __nv_bfloat16* a4 = nullptr;        // [n][14][128] conv3 outputs
   CUtensorMap mapA, mapB;             // TMA maps of a4 [n][1792] and wfc1 [256][1792]
+  CUtensorMap mapB128;                // wfc1 with a 128-row box (fc1_head pair mode)
+  bool pair = false;                  // fc1_head on 2-SM MMAs (PSIM_FC1_PAIR)
   int grid_cap = 0;                   // max CTAs of the persistent fused kernels (0: one per SM);
                                       // cohorts with disjoint SM shares run side by side
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)

@@ -753,6 +753,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
   if (predict && !fused) { rc = ensure_buffers(ctx, std::max<uint64_t>(n, 1)); if (rc) return rc; }
   if (fused) {
     FusedC3& fz = ctx->fused;
+    fz.pair = (ctx->opts.flags & PSIM_FC1_PAIR) != 0;
     const uint64_t nn = std::max<uint64_t>(n, 1);
     if (fz.cap_n != nn) {
       dfree(fz.blocks); dfree(fz.count); dfree(fz.tileP[0]); dfree(fz.tileP[1]); dfree(fz.a4);

@@ -28,10 +28,11 @@ def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, 
     """variant (teacher-forced runs): "warp" = the standalone warp-per-sub-trace update
     kernel; "fused" = the thread-per-sub-trace update inside fc1_head_kernel (the hot
     path), reached by running the fused C3 CNN with PSIM_FORCE_PREDICT while the queue
-    follows the forced latencies."""
-    fused_forced = forced is not None and variant == "fused"
+    follows the forced latencies; "pair" = the same with fc1_head on 2-SM MMAs."""
+    fused_forced = forced is not None and variant in ("fused", "pair")
     with P.Simulator(precision="bf16" if fused_forced else precision, queue_cap=cap, record_rows=record, rank=rank,
-                     world_size=world, layerwise=layerwise, force_predict=fused_forced) as sim:
+                     world_size=world, layerwise=layerwise, force_predict=fused_forced,
+                     fc1_pair=variant == "pair") as sim:
         if device_trace:
             t = torch.from_numpy(np.ascontiguousarray(trace)).cuda()
             sim.load_trace(t, n_instr=n_instr, first_row=first_row)
@@ -56,7 +57,7 @@ def gpu_run(trace, N, W, *, arch="C3", weights=None, precision="bf16", cap=110, 
 
 
 # ------------------------------------------------------------------ S1
-VARIANTS = ["warp", "fused"]
+VARIANTS = ["warp", "fused", "pair"]   # pair: fused with fc1_head on 2-SM MMAs (PSIM_FC1_PAIR)
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -470,8 +471,8 @@ def test_fused_deterministic_many_tiles():
     w = synth.weights("C3")
     pinned = torch.from_numpy(tr).pin_memory()
     runs = []
-    for src in ("device", "device", "pinned"):
-        with P.Simulator(precision="bf16") as sim:
+    for src, pair in (("device", False), ("device", False), ("pinned", False), ("device", True)):
+        with P.Simulator(precision="bf16", fc1_pair=pair) as sim:   # pair: fc1_head on 2-SM MMAs
             sim.load_trace(torch.from_numpy(tr).cuda() if src == "device" else pinned)
             sim.partition(N, W)
             sim.load_model("C3", w)
