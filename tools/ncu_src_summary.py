@@ -4,7 +4,8 @@
 
 Maps the SASS offsets of the report's source page to CUDA source lines with the line table
 of the in-tree libpsim.so (nvdisasm --print-line-info; the .so must be the build that was
-profiled) and prints the lines with the most stall samples and their top stall reasons."""
+profiled; PSIM_LIB / PSIM_CSRC point at another build and its sources) and prints the lines with
+the most stall samples and their top stall reasons."""
 import collections
 import csv
 import io
@@ -15,11 +16,11 @@ import sys
 import tempfile
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-CSRC = os.path.join(ROOT, "paper_conf_sc_pandeylfhl22_b200", "csrc")
+CSRC = os.environ.get("PSIM_CSRC") or os.path.join(ROOT, "paper_conf_sc_pandeylfhl22_b200", "csrc")
 
 
 def line_table(kern):
-    lib = os.path.join(ROOT, "paper_conf_sc_pandeylfhl22_b200", "libpsim.so")
+    lib = os.environ.get("PSIM_LIB") or os.path.join(ROOT, "paper_conf_sc_pandeylfhl22_b200", "libpsim.so")
     with tempfile.TemporaryDirectory() as d:
         subprocess.run(["cuobjdump", "-xelf", "all", lib], cwd=d, capture_output=True, check=True)
         sass = ""
@@ -31,8 +32,8 @@ def line_table(kern):
     start = [i for i, l in enumerate(lines) if l.startswith(".text._ZN4psim") and kern in l][0]
     off2line, cur = {}, None
     for l in lines[start + 1:]:
-        if l.startswith(".text."):
-            break
+        if l.startswith(".text.") or l.startswith("//---") or l.lstrip().startswith(".section"):
+            break                                   # next function / section / cubin
         m = re.search(r'//## File "([^"]+)", line (\d+)', l)
         if m:
             cur = (os.path.basename(m.group(1)), int(m.group(2)))
