@@ -48,11 +48,13 @@ constexpr int W1_OFF = 0;                    // 2 atoms [64][64]   8 KB each
 constexpr int W2_OFF = W1_OFF + 16 * 1024;   // 2 atoms [128][64] 16 KB each
 constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of W3, streamed by TMA
                                              // (halves alternate with the conv3 MMAs, from L2)
-constexpr int NX = 3;                        // X slots: gathered items in flight
+constexpr int NX = 2;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
 constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][128 B] (half rows)
 constexpr int BE_OFF = STG_OFF + 16 * 1024;  // uint4 [3 tiles][256 issuer lanes]: block entries staged by cp.async
-constexpr int BAR_OFF = BE_OFF + 12 * 1024;  // mbarriers
+constexpr int ER = 8, ED = 4;                // queue-entry ring: items staged ED ahead in ER slots
+constexpr int ER_OFF = BE_OFF + 12 * 1024;   // uint4 [ER items][256 issuer lanes]: queue entries staged by cp.async
+constexpr int BAR_OFF = ER_OFF + ER * 4096;  // mbarriers
 constexpr int BIAS_OFF = BAR_OFF + 512;      // b1[64] b2[128] b3[128] fp32
 constexpr int SMEM = BIAS_OFF + 1280 + 1024; // + alignment slack (<= 227 KB)
 static_assert(SMEM <= 232448, "conv_stack smem over the 227 KB opt-in limit");
@@ -451,20 +453,14 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     const uint64_t pol = l2_policy_evict_first();
     const uint4 kNoBlock = make_uint4(0xFFFFFFFFu, 0u, 0u, 0u);
     auto row_R = [&](const uint4& be, uint32_t n) -> int { return (int)(be.x & 15) * 8 + 2 * (int)(n & 3) + hh; };
-    auto load_entry = [&](const uint4& be, uint32_t n) -> uint4 {   // queue entry of this lane's row of item n
-      const int R = row_R(be, n), k = (int)be.y;
-      if (be.x == 0xFFFFFFFFu || R < 1 || R > k) return make_uint4(0, 0, 0, 0);
-      return __ldcg(a.q + (uint64_t)(k - R) * a.qn + (be.x >> 4));
-    };
-    // Metadata pipeline: block entries of tiles T and T + 1 in registers (from smem); the
-    // queue entry of item n + 4 is prefetched into L2 (no register) and loaded into
-    // registers at item n + 2 (evA / evB by item parity), so neither the DRAM nor the L2
-    // latency of the step's loaded memory system sits on the issue path.  The loop is
-    // unrolled by two so a pending load is never the source of a register move (a move
-    // would wait for the load).
-    // block entries of tile T live in smem slot T % 3 (lane-private), staged by cp.async two
-    // tiles ahead; beC / beN are register copies of tiles T / T + 1 read at each tile start
+    // Metadata pipeline, all through lane-private smem rings filled by cp.async (no register
+    // ever waits on a load in flight): block entries of tile T in slot T % 3, staged two
+    // tiles ahead (beC / beN = register copies of tiles T / T + 1 read at each tile start);
+    // the queue entry of item n in slot n % ER, staged ED items ahead.  One cp.async group
+    // per item (its entry) and one per tile (a block-entry slot): the wait before item n
+    // allows the ED - 1 later entry groups (+ at most one block-entry group) to stay pending.
     uint4* sBE = reinterpret_cast<uint4*>(sm + cs::BE_OFF) + wq * 32 + lane;
+    uint4* sER = reinterpret_cast<uint4*>(sm + cs::ER_OFF) + wq * 32 + lane;
     auto stage_block = [&](uint32_t T) {
       const uint32_t bi = (blockIdx.x + T * gridDim.x) * cs::TILE + m;
       uint4* dst = sBE + (T % 3) * 256;
@@ -472,27 +468,29 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       else *dst = kNoBlock;
       cp_async_commit();
     };
+    const uint32_t n_items = my_tiles * 4;
+    auto stage_entry = [&](const uint4& be, uint32_t n) {   // queue entry of this lane's row of item n
+      const int R = row_R(be, n), k = (int)be.y;
+      if (n < n_items && be.x != 0xFFFFFFFFu && R >= 1 && R <= k)
+        cp_async16(sER + (n % cs::ER) * 256, a.q + (uint64_t)(k - R) * a.qn + (be.x >> 4));
+      cp_async_commit();
+    };
     stage_block(0);
     stage_block(1);
     cp_async_wait<0>();
     uint4 beC = sBE[0], beN = sBE[256];
-    stage_block(2);
-    const uint32_t n_items = my_tiles * 4;
-    auto entry_ptr = [&](const uint4& be, uint32_t n) -> const uint4* {   // nullptr: no queue entry
-      const int R = row_R(be, n), k = (int)be.y;
-      if (be.x == 0xFFFFFFFFu || R < 1 || R > k) return nullptr;
-      return a.q + (uint64_t)(k - R) * a.qn + (be.x >> 4);
-    };
-    constexpr bool kPrefetchL2 = false;   // L2 prefetch of item n + 4's entry: measured slower (LSU pressure)
 #pragma unroll
-    for (uint32_t n = 2; n < 4; ++n)
-      if (kPrefetchL2)
-        if (const uint4* p = entry_ptr(beC, n)) prefetch_l2(p);
-    uint4 evA = load_entry(beC, 0), evB = load_entry(beC, 1);
-    auto item = [&](uint32_t nI, uint4& ev) {
+    for (uint32_t n = 0; n < (uint32_t)cs::ED; ++n) stage_entry(beC, n);   // ED == 4: tile 0
+    stage_block(2);
+    // commit order ... E(n) E(n+1) E(n+2) E(n+3) with exactly one block-entry group among
+    // the four groups after any E(n), and exactly four entry groups after BE(T + 2) at the
+    // end of tile T: cp.async.wait_group 4 is exact in both places
+    static_assert(cs::ED == 4 && cs::ER >= 2 * cs::ED, "entry ring: items n + ED stay in tile + 1");
+    auto item = [&](uint32_t nI) {
       const uint32_t it = nI >> 2;                     // this CTA's tile of item nI
       [[maybe_unused]] const int j = (int)(nI & 3);    // conv1 position (timestamps)
       if (warp == cs::GATHER_WARP0) PSIM_TS(81 + 3 * j);
+      cp_async_wait<cs::ED>();                         // item nI's entry has landed (own slot)
       // ---- build this lane's row of item nI
       uint32_t row;
       uint2 tc = make_uint2(0u, 0u);
@@ -503,6 +501,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         } else if (R == 0) {
           row = (uint32_t)((int64_t)(beC.z + (uint32_t)a.step) - a.row_lo);   // current instruction first
         } else {
+          const uint4 ev = sER[(nI % cs::ER) * 256];
           const int c = ev.z & 0xFFFF, sv = (ev.z >> 16) & 0xFFFF;
           const int age = (int)(beC.w - ev.y);
           const int t0 = min(age, kTimeMax), t1 = min(max(0, c - age), kTimeMax), t2 = min(c + sv - age, kTimeMax);
@@ -511,12 +510,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         }
       }
       if (warp == cs::GATHER_WARP0) PSIM_TS(83 + 3 * j);
-      // the entry of item nI + 2 (tile it or it + 1) into the same registers; item nI + 4
-      // (tile it + 1) into L2
-      const uint32_t n2 = nI + 2;
-      ev = (n2 < n_items) ? load_entry((n2 >> 2) == it ? beC : beN, n2) : make_uint4(0, 0, 0, 0);
-      if (kPrefetchL2 && nI + 4 < n_items)
-        if (const uint4* p = entry_ptr(beN, nI + 4)) prefetch_l2(p);
+      stage_entry(beN, nI + cs::ED);                   // item nI + 4: tile it + 1
       if (warp == cs::GATHER_WARP0) PSIM_TS(97 + 2 * j);
       // row indices of the 4 blocks this lane gathers (TMA lanes 0..7): lanes 4 g + i + 16 h
       const uint32_t r0 = __shfl_sync(0xffffffffu, row, 4 * g + 0 + 16 * h);
@@ -543,17 +537,15 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       __syncwarp();
       if (warp == cs::GATHER_WARP0) PSIM_TS(96 + 2 * j);
       if (((nI + 1) & 3) == 0) {                        // the next item starts tile it + 1
-        cp_async_wait<0>();                             // tile it + 2's entries (staged a tile ago)
+        cp_async_wait<4>();                             // tile it + 2's block entries (staged a tile ago;
+                                                        // only this tile's 4 entry groups are younger)
         beC = beN;
         beN = sBE[((it + 2) % 3) * 256];
         stage_block(it + 3);                            // into slot it % 3 (tile it is done)
       }
     };
 #pragma unroll 1
-    for (uint32_t nI = 0; nI < n_items; nI += 2) {      // n_items is a multiple of 4
-      item(nI, evA);
-      item(nI + 1, evB);
-    }
+    for (uint32_t nI = 0; nI < n_items; ++nI) item(nI);
   }
   fence_before();
   __syncthreads();
