@@ -76,6 +76,11 @@ static_assert(2 * REG_EPI + REG_MMA + 2 * REG_ISSUE <= THREADS * 96 / 128, "setm
 
 }  // namespace cs
 
+// Epilogue split (experiment): EG-B's conv3 epilogue (TMEM -> bias, ReLU, bf16 -> staged, coalesced a4
+// stores) takes about as long as a whole tile, so the conv2 position-1 epilogue runs on EG-A
+// (after its conv1 epilogues of the tile) instead of EG-B
+constexpr bool kEgaConv2Pos1 = false;   // measured neutral (A/B 554.5 vs 555.2 MIPS, G=8 238.2 vs 239.1)
+
 struct ConvArgs {
   const uint4* blocks;       // block entries {b << 4 | p, k, ws lo, Clock lo} of this step
   const uint32_t* nblocks;   // count of this step's list
@@ -347,10 +352,10 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(a2full + s);
         if (q == 0) PSIM_TS(48 + j);
-        if (j == 1) {   // conv2 position 0 (items 0 and 1) is complete after conv2 MMAs (0, *)
-          if (q == 0) PSIM_TS(56);
-          conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, 0, lane);
-          if (q == 0) PSIM_TS(59);
+        if (j == 1 || (kEgaConv2Pos1 && j == 3)) {   // conv2 position j / 2 (items j - 1, j) after conv2 MMAs (j / 2, *)
+          if (q == 0) PSIM_TS(j == 1 ? 56 : 60);
+          conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, j >> 1, lane);
+          if (q == 0) PSIM_TS(j == 1 ? 59 : 63);
         }
       }
     }
@@ -415,9 +420,11 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     uint32_t it = 0, prev_tl = 0;
     for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x, ++it) {
       if (it > 0) e3(it - 1, prev_tl);
-      if (q == 0) PSIM_TS(60);
-      conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, 1, lane);
-      if (q == 0) PSIM_TS(63);
+      if constexpr (!kEgaConv2Pos1) {
+        if (q == 0) PSIM_TS(60);
+        conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, 1, lane);
+        if (q == 0) PSIM_TS(63);
+      }
       prev_tl = tl;
     }
     if (it > 0) e3(it - 1, prev_tl);
