@@ -1101,8 +1101,10 @@ static void launch_pdl(void (*kern)(KArgs...), int grid, int threads, int smem, 
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
+  // PSIM_NO_PDL=1 (experiments): plain stream-ordered launches; griddepcontrol.wait is then a no-op
+  static const bool no_pdl = [] { const char* e = getenv("PSIM_NO_PDL"); return e && atoi(e) != 0; }();
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = no_pdl ? 0 : 1;
   cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
