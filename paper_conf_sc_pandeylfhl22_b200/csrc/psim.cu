@@ -621,12 +621,26 @@ static int run_cnn(psim_ctx* ctx, uint64_t n) {
   const bool bf16 = m.precision == PSIM_BF16;
   const void* in = ctx->buf.x;
   const void* block_in = nullptr;
+  // RB7 residual blocks fused into one kernel each (resblock.cu; PSIM_RB7_FUSED=0: layer-wise A/B)
+  static const bool rb7_fused = [] { const char* e = getenv("PSIM_RB7_FUSED"); return !(e && atoi(e) == 0); }();
   for (size_t li = 0; li < m.layers.size(); ++li) {
     const GemmLayer& g = m.layers[li];
     const bool last = li + 1 == m.layers.size();
     void* out = last ? (void*)ctx->buf.h : ctx->buf.act[li];
     const int64_t M = (int64_t)n * g.rows_per_item;
     if (g.block_begin) block_in = in;
+    if (bf16 && rb7_fused && g.block_begin && g.taps == 3 && li + 1 < m.layers.size() && g.N == 64 && g.K == 192 &&
+        m.layers[li + 1].add_block_input && m.layers[li + 1].taps == 3 && !g.w_sp) {
+      const GemmLayer& gb = m.layers[li + 1];
+      void* outb = ctx->buf.act[li + 1];
+      pf.begin(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
+      launch_resblock((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w, g.bias, (const __nv_bfloat16*)gb.w, gb.bias,
+                      (__nv_bfloat16*)outb, M, ctx->stream);
+      pf.end(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
+      in = outb;
+      ++li;   // conv_b done inside the block kernel
+      continue;
+    }
     pf.begin(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
     if (bf16 && g.w_sp) {   // 2:4 structured-sparse tcgen05.mma.sp (PSIM_SPARSE24)
       launch_gemm_sp((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w_sp, g.meta, g.sp_mh, g.bias, out, last, M,
