@@ -25,50 +25,76 @@ __device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a,
 }
 
 // X[b][r][c]: row 0 = current instruction (time columns 0), rows 1..k = live
-// entries newest first (R6), rows > k zero (PAPER.md:93 zero padding).
-// Lane l writes columns 2l, 2l+1.
+// entries newest first (R6), rows > k zero (PAPER.md:93 zero padding); the item's
+// extra pad rows (RB7 layout: item_rows = 116, row_off = 2) are zero.
+// Eight threads per (sub-trace, item row), thread c of a row building features 8c .. 8c + 7:
+// the whole input of a sub-trace is built in parallel (independent loads of the queue entry
+// and of two aligned 8-byte words of the trace row), and a warp stores four consecutive
+// rows as one contiguous 512-byte (bf16) / 1 KB (fp32) span.
 template <typename T>
 __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict__ x) {
-  const int lane = threadIdx.x & 31;
-  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = (gridDim.x * (uint64_t)blockDim.x) >> 5;
-  const int c0 = 2 * lane, c1 = 2 * lane + 1;
-  for (uint64_t b = warp; b < a.n; b += nwarps) {
+  const uint64_t total = a.n * (uint64_t)a.item_rows * 8;
+  const bool aligned8 = ((a.stride | reinterpret_cast<uintptr_t>(a.trace)) & 7) == 0;
+  for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < total; t += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t rr = t >> 3;                                        // global item row
+    const int ch = (int)(t & 7);                                       // 8-feature chunk of the row
+    const uint64_t b = rr / (uint64_t)a.item_rows;
+    const int r = (int)(rr - b * (uint64_t)a.item_rows) - a.row_off;  // input row (PAPER.md:93 order)
     const int64_t ws = a.ws[b];
-    if (a.step >= a.e[b] - ws) continue;                      // sub-trace finished
-    const int64_t i = ws + a.step;
+    if (a.step >= a.e[b] - ws) continue;                               // sub-trace finished
     const int k = a.count[b];
-    const uint32_t clo = (uint32_t)a.clock[b];
-    T* xb = x + (b * (uint64_t)a.item_rows + a.row_off) * kFeatPad;
-    const uint4* qb = a.q + b;             // entry-major: entry e at [e * n]
-    for (int r = 0; r < kRows; ++r) {
-      float v0 = 0.f, v1 = 0.f;
-      if (r <= k) {
-        int64_t row;
-        int age = 0, remc = 0, remr = 0;
-        if (r == 0) {
-          row = i;
-        } else {
-          const int ent = k - r;                                  // newest first
-          const uint4 en = qb[ent * a.n];
-          row = en.x;
-          const uint32_t cs = en.z;
-          const int c = cs & 0xFFFF, s = cs >> 16;
-          age = (int)(clo - en.y);
-          remc = max(0, c - age);
-          remr = c + s - age;
-          age = min(age, kTimeMax); remc = min(remc, kTimeMax); remr = min(remr, kTimeMax);
+    float v[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) v[c] = 0.f;
+    if (r >= 0 && r <= k && r < kRows && ch < 7) {                    // features 56..63 are zero
+      int64_t row;
+      if (r == 0) {
+        row = ws + a.step;                                             // current instruction first
+      } else {
+        const uint4 en = a.q[(uint64_t)(k - r) * (a.qn ? a.qn : a.n) + b];   // newest first (R6)
+        row = en.x;
+        if (ch == 0) {                                                 // R2 time features, clamped (R7)
+          const uint32_t clo = (uint32_t)a.clock[b];
+          const int c = en.z & 0xFFFF, s = en.z >> 16;
+          const int age = (int)(clo - en.y);
+          v[0] = (float)min(age, kTimeMax);
+          v[1] = (float)min(max(0, c - age), kTimeMax);
+          v[2] = (float)min(c + s - age, kTimeMax);
         }
-        const uint8_t* ar = a.trace + (row - a.row_lo) * a.stride;
-        auto col = [&](int c) -> float {
-          if (c < 3) return c == 0 ? (float)age : (c == 1 ? (float)remc : (float)remr);
-          if (c < kFeat) return (float)__ldg(ar + (c - 3));
-          return 0.f;
-        };
-        v0 = col(c0);
-        v1 = col(c1);
       }
-      store2<T>(xb + r * kFeatPad + c0, v0, v1);
+      // feature f = 8 ch + i (i < 8) is attribute f - 3 for 3 <= f < 50: trace bytes 8 ch - 3 .. 8 ch + 4
+      const uint8_t* ar = a.trace + (row - a.row_lo) * a.stride;
+      if (aligned8) {
+        const uint2 lo = ch > 0 ? __ldg(reinterpret_cast<const uint2*>(ar) + ch - 1) : make_uint2(0u, 0u);
+        const uint2 hi = __ldg(reinterpret_cast<const uint2*>(ar) + ch);   // bytes 8 ch .. 8 ch + 7
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int f = 8 * ch + i;
+          if (f < 3 || f >= kFeat) continue;
+          const int byte = f - 3 - 8 * (ch - 1);                       // offset within [lo | hi]
+          const uint32_t w = byte < 4 ? lo.x : byte < 8 ? lo.y : byte < 12 ? hi.x : hi.y;
+          v[i] = (float)((w >> ((byte & 3) * 8)) & 0xFFu);
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int f = 8 * ch + i;
+          if (f >= 3 && f < kFeat) v[i] = (float)__ldg(ar + (f - 3));
+        }
+      }
+    }
+    T* xr = x + rr * kFeatPad + 8 * ch;
+    if constexpr (sizeof(T) == 2) {
+      uint32_t p[4];
+#pragma unroll
+      for (int h = 0; h < 4; ++h) {
+        __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * h], v[2 * h + 1]);   // RNE (oracle bf16 mode)
+        p[h] = *reinterpret_cast<uint32_t*>(&h2);
+      }
+      *reinterpret_cast<uint4*>(xr) = make_uint4(p[0], p[1], p[2], p[3]);
+    } else {
+      reinterpret_cast<float4*>(xr)[0] = make_float4(v[0], v[1], v[2], v[3]);
+      reinterpret_cast<float4*>(xr)[1] = make_float4(v[4], v[5], v[6], v[7]);
     }
   }
 }
@@ -80,11 +106,16 @@ static int grid_for(uint64_t warps, int block = 256) {
   return (int)blocks;
 }
 
+static int grid_rows(uint64_t rows) {   // threads -> CTAs of 256, at most 148 x 16
+  uint64_t blocks = (rows + 255) / 256;
+  if (blocks > 148ull * 16) blocks = 148ull * 16;
+  return (int)std::max<uint64_t>(blocks, 1);
+}
 void launch_gather_f32(const GatherArgs& a, float* x, cudaStream_t st) {
-  gather_kernel<float><<<grid_for(a.n), 256, 0, st>>>(a, x);
+  gather_kernel<float><<<grid_rows(a.n * (uint64_t)a.item_rows * 8), 256, 0, st>>>(a, x);
 }
 void launch_gather_bf16(const GatherArgs& a, __nv_bfloat16* x, cudaStream_t st) {
-  gather_kernel<__nv_bfloat16><<<grid_for(a.n), 256, 0, st>>>(a, x);
+  gather_kernel<__nv_bfloat16><<<grid_rows(a.n * (uint64_t)a.item_rows * 8), 256, 0, st>>>(a, x);
 }
 
 // ---------------------------------------------------------------------------
