@@ -9,10 +9,12 @@
 // sub-traces -- 2 x 58 pad-row positions = 116 rows of the [n * 58][64] activation, padded
 // to the MMA's M = 128 -- is self-contained: each sub-trace's pad rows (positions 0 and 57,
 // kept zero) are exactly the zero padding of both convolutions, so the halo never leaves the
-// tile.  conv_a's three taps are TMA loads of the input rows shifted by -1 / 0 / +1 (rows
-// outside the tensor read as zero); its ReLU'd output is written by the epilogue into three
-// row-shifted copies in shared memory that are conv_b's three A operands; the residual x is
-// the unshifted tap tile still in shared memory.  Only x is read and y written per block.
+// tile.  One TMA load brings the tile's 130 input rows (r0 - 1 .. r0 + 128; rows outside the
+// tensor read as zero); conv_a's three taps are SWIZZLE_128B descriptors of that tile starting
+// at rows 0 / 1 / 2 (a descriptor may start at any 128-B row: the swizzle follows the address,
+// tools/gpu/exp/rowshift_probe.cu); its ReLU'd output goes into one 130-row buffer (row m + 1)
+// whose row-shifted descriptors are conv_b's taps; the residual x is the input tile's row
+// m + 1.  Only x is read and y written per block; ~100 KB of smem: two CTAs per SM.
 //
 // Roles (320 threads): warp 0 TMA producer (weights once, then the 3 tap tiles per tile,
 // two stages), warp 1 TMEM allocator + MMA issuer (order a(0) a(1) b(0) a(2) b(1) ...: the
@@ -33,17 +35,19 @@ using namespace tc;
 namespace rb {
 constexpr int P = 58;                        // pad-row positions per sub-trace (56 + 2)
 constexpr int TROWS = 2 * P;                 // tile rows that are real (two sub-traces)
+constexpr int XROWS = 130;                   // a tile's input rows r0 - 1 .. r0 + 128 (the taps' halo)
+constexpr int XSTAGE = 17 * 1024;            // one SW128 tile of 130 rows x 128 B (1024-aligned stages)
 constexpr int W_OFF = 0;                     // W_a, W_b: [64 N][192 K] bf16 as 3 K-atoms of [64][64] each
-constexpr int X_OFF = 48 * 1024;             // 2 stages x 3 tap tiles [128][64] bf16 (16 KB each)
-constexpr int ACT_OFF = X_OFF + 2 * 48 * 1024;   // 3 row-shifted copies of relu(conv_a) [128][64]
-constexpr int BIAS_OFF = ACT_OFF + 48 * 1024;    // b_a[64], b_b[64] fp32
+constexpr int X_OFF = 48 * 1024;             // 2 stages
+constexpr int ACT_OFF = X_OFF + 2 * XSTAGE;  // relu(conv_a) at rows 1..128 (row 0 and 129 zero)
+constexpr int BIAS_OFF = ACT_OFF + XSTAGE;   // b_a[64], b_b[64] fp32
 constexpr int BAR_OFF = BIAS_OFF + 512;
-constexpr int SMEM = BAR_OFF + 256 + 1024;
+constexpr int SMEM = BAR_OFF + 256 + 1024;   // ~100 KB: two CTAs per SM
 constexpr int THREADS = 320;                 // warp 0 TMA, 1 MMA, 2..5 epilogue A, 6..9 epilogue B
 }  // namespace rb
 static_assert(rb::SMEM <= 232448, "resblock smem over the 227 KB opt-in limit");
 
-__global__ void __launch_bounds__(rb::THREADS, 1)
+__global__ void __launch_bounds__(rb::THREADS, 2)
     resblock_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmWa,
                     const __grid_constant__ CUtensorMap tmWb, const float* __restrict__ ba,
                     const float* __restrict__ bb, __nv_bfloat16* __restrict__ y, int64_t M) {
@@ -93,10 +97,11 @@ __global__ void __launch_bounds__(rb::THREADS, 1)
       for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
         const int s = it & 1;
         wait_empty(xempty + s, it >> 1);
-        mbar_expect_tx(xfull + s, 3 * 16384);
-        const int r0 = (int)(tile * rb::TROWS);
-        for (int t = 0; t < 3; ++t)   // tap t reads input row r + t - 1 (row -1 / M.. zero-filled)
-          tma_load_2d(sm + rb::X_OFF + s * 49152 + t * 16384, &tmX, xfull + s, 0, r0 + t - 1);
+        mbar_expect_tx(xfull + s, rb::XROWS * 128);
+        // rows r0 - 1 .. r0 + 128 (row -1 / rows >= M zero-filled): tap t of output row m reads
+        // smem row m + t, so the three taps are row-shifted descriptors of this one tile (a
+        // SWIZZLE_128B descriptor may start at any 128-B row: the swizzle follows the address)
+        tma_load_2d(sm + rb::X_OFF + s * rb::XSTAGE, &tmX, xfull + s, 0, (int)(tile * rb::TROWS) - 1);
       }
     }
   } else if (warp == 1) {
@@ -111,7 +116,7 @@ __global__ void __launch_bounds__(rb::THREADS, 1)
         fence_after();
         for (int t = 0; t < 3; ++t)
           for (int k = 0; k < 4; ++k)
-            mma_bf16(tmem + s * 64, sw128_desc(sbase + rb::X_OFF + s * 49152 + t * 16384 + 32 * k),
+            mma_bf16(tmem + s * 64, sw128_desc(sbase + rb::X_OFF + s * rb::XSTAGE + t * 128 + 32 * k),
                      sw128_desc(sbase + rb::W_OFF + t * 8192 + 32 * k), idesc, (t | k) != 0);
         mma_commit(dafull + s);
       };
@@ -122,7 +127,7 @@ __global__ void __launch_bounds__(rb::THREADS, 1)
         fence_after();
         for (int t = 0; t < 3; ++t)
           for (int k = 0; k < 4; ++k)
-            mma_bf16(tmem + 128 + s * 64, sw128_desc(sbase + rb::ACT_OFF + t * 16384 + 32 * k),
+            mma_bf16(tmem + 128 + s * 64, sw128_desc(sbase + rb::ACT_OFF + t * 128 + 32 * k),
                      sw128_desc(sbase + rb::W_OFF + 24576 + t * 8192 + 32 * k), idesc, (t | k) != 0);
         mma_commit(actempty);
         mma_commit(dbfull + s);
@@ -167,17 +172,14 @@ __global__ void __launch_bounds__(rb::THREADS, 1)
         for (int c = 0; c < 32; ++c) pk[c] = 0u;
       wait_empty(actempty, it);                            // conv_b of the previous tile done with them
       uint8_t* act = sm + rb::ACT_OFF;
-      // copy t row m' holds activation row m' + t - 1: row m goes to copy 0 row m + 1, copy 1
-      // row m, copy 2 row m - 1; copy 0 row 0 = row -1 of the tile = the previous tile's last
-      // pad row (zero); copy 2 row 127 feeds only junk rows
+      // activation row m at buffer row m + 1: conv_b's tap t of output row m reads buffer row
+      // m + t = activation row m + t - 1; row 0 (activation row -1 = the previous tile's last pad
+      // row) is zero, row 129 feeds only junk rows
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
-        const uint4 v = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
-        st_sw128(act + 16384, m, c, v);
-        if (m + 1 < 128) st_sw128(act, m + 1, c, v);
-        if (m >= 1) st_sw128(act + 32768, m - 1, c, v);
+        st_sw128(act, m + 1, c, make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]));
         if (m == 0) st_sw128(act, 0, c, make_uint4(0, 0, 0, 0));
-        if (m == 127) st_sw128(act + 32768, 127, c, make_uint4(0, 0, 0, 0));
+        if (m == 127) st_sw128(act, 129, c, make_uint4(0, 0, 0, 0));
       }
       fence_async_smem();                                  // visible to the tensor core
       __syncwarp();
@@ -187,34 +189,29 @@ __global__ void __launch_bounds__(rb::THREADS, 1)
       // ---- B: relu(conv_b + b_b + x) -> y
       wait_full(dbfull + s, it >> 1);
       fence_after();
-      {
-        uint32_t r0[32], r1[32];
-        tmem_ld32_nowait(tmem + lane_base + 128 + s * 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + 128 + s * 64 + 32, r1);
-        tmem_wait_ld();
-        fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(dbempty + s);
-        // residual: the unshifted tap tile (tap 1) row m, read back from its swizzled layout
-        const uint8_t* xt = sm + rb::X_OFF + s * 49152 + 16384;
-        uint32_t xv[32];
+      const uint8_t* xt = sm + rb::X_OFF + s * rb::XSTAGE;   // residual x row m = tile row m + 1
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-          const uint4 u = *reinterpret_cast<const uint4*>(xt + m * 128 + ((c ^ (m & 7)) << 4));
+      for (int hf = 0; hf < 2; ++hf) {                      // channels 32 hf .. 32 hf + 31 (register budget)
+        uint32_t r0[32];
+        tmem_ld32_nowait(tmem + lane_base + 128 + s * 64 + 32 * hf, r0);
+        tmem_wait_ld();
+        uint32_t xv[16];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          const int cc = 4 * hf + c;
+          const uint4 u = *reinterpret_cast<const uint4*>(xt + (m + 1) * 128 + ((cc ^ ((m + 1) & 7)) << 4));
           xv[4 * c] = u.x; xv[4 * c + 1] = u.y; xv[4 * c + 2] = u.z; xv[4 * c + 3] = u.w;
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(xempty + s);           // the X stage may be refilled
 #pragma unroll
-        for (int c = 0; c < 16; ++c) {                     // channels 2c, 2c+1 (r0) and 32 + 2c, 33 + 2c (r1)
+        for (int c = 0; c < 16; ++c) {                      // channels 32 hf + 2c, + 1
           const float x0 = __uint_as_float(xv[c] << 16), x1 = __uint_as_float(xv[c] & 0xFFFF0000u);
-          const float x2 = __uint_as_float(xv[16 + c] << 16), x3 = __uint_as_float(xv[16 + c] & 0xFFFF0000u);
-          pk[c] = pack_bf16_relu(__uint_as_float(r0[2 * c]) + sbias[64 + 2 * c] + x0,
-                                 __uint_as_float(r0[2 * c + 1]) + sbias[65 + 2 * c] + x1);
-          pk[16 + c] = pack_bf16_relu(__uint_as_float(r1[2 * c]) + sbias[96 + 2 * c] + x2,
-                                      __uint_as_float(r1[2 * c + 1]) + sbias[97 + 2 * c] + x3);
+          pk[16 * hf + c] = pack_bf16_relu(__uint_as_float(r0[2 * c]) + sbias[64 + 32 * hf + 2 * c] + x0,
+                                           __uint_as_float(r0[2 * c + 1]) + sbias[65 + 32 * hf + 2 * c] + x1);
         }
       }
+      fence_before();
+      __syncwarp();
+      if (lane == 0) { mbar_arrive(dbempty + s); mbar_arrive(xempty + s); }   // accumulator drained, X stage free
       if (m < rb::TROWS && row < M) {
         uint4* dst = reinterpret_cast<uint4*>(y + row * 64);
 #pragma unroll
@@ -266,13 +263,13 @@ void launch_resblock(const __nv_bfloat16* x, const __nv_bfloat16* wa, const floa
     attr = true;
   }
   CUtensorMap mx, mwa, mwb;
-  if (M % rb::P != 0 || !map_rb(&mx, x, (uint64_t)M, 64, 128) || !map_rb(&mwa, wa, 64, 192, 64) ||
+  if (M % rb::P != 0 || !map_rb(&mx, x, (uint64_t)M, 64, rb::XROWS) || !map_rb(&mwa, wa, 64, 192, 64) ||
       !map_rb(&mwb, wb, 64, 192, 64)) {
     cudaLaunchKernel((const void*)nullptr, dim3(1), dim3(1), nullptr, 0, st);   // error for the caller
     return;
   }
   const int64_t tiles = (M + rb::TROWS - 1) / rb::TROWS;
-  const int grid = (int)std::min<int64_t>(tiles, (int64_t)sm_count());
+  const int grid = (int)std::min<int64_t>(tiles, 2 * (int64_t)sm_count());   // two CTAs per SM
   resblock_kernel<<<grid, rb::THREADS, rb::SMEM, st>>>(mx, mwa, mwb, ba, bb, y, M);
 }
 
