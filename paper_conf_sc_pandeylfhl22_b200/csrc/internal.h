@@ -189,6 +189,10 @@ int sparse24_compress(const uint16_t* W, int N, int K, std::vector<uint16_t>* wc
 // C[M][N] = act(X[M][K] . W^T + b) with W 2:4-sparse (compressed + metadata from sparse24_compress)
 void launch_gemm_sp(const __nv_bfloat16* X, const __nv_bfloat16* Wc, const uint32_t* meta, int mh, const float* b,
                     void* C, bool c_is_f32, int64_t M, int N, int K, bool relu, cudaStream_t st);
+// RB7 gather + stem convolution fused on tcgen05 (rb7_stem.cu): the step's inputs built straight
+// into the stem's A operand; y = the stem output in the pad-row layout [n * 58][64] bf16
+void launch_rb7_stem(const GatherArgs& g, const __nv_bfloat16* w, const float* bias, __nv_bfloat16* y,
+                     cudaStream_t st);
 // RB7 residual block fused on tcgen05 (resblock.cu): y = relu(x + conv_b(relu(conv_a(x)))) over the
 // pad-row layout [M = n * 58][64] bf16; wa / wb: [64][192] bf16 (K = tap * 64 + channel)
 void launch_resblock(const __nv_bfloat16* x, const __nv_bfloat16* wa, const float* ba, const __nv_bfloat16* wb,

@@ -615,15 +615,16 @@ static int ensure_buffers(psim_ctx* ctx, uint64_t n) {
 }
 
 // Run the lowered CNN on buf.x (n items) -> buf.y.  Counts launches.
-static int run_cnn(psim_ctx* ctx, uint64_t n) {
+// layers [first, end) of the lowered CNN on `in0` (default: the gathered inputs buf.x)
+static int run_cnn(psim_ctx* ctx, uint64_t n, size_t first = 0, const void* in0 = nullptr) {
   const Model& m = ctx->model;
   Prof& pf = ctx->prof;
   const bool bf16 = m.precision == PSIM_BF16;
-  const void* in = ctx->buf.x;
+  const void* in = in0 ? in0 : ctx->buf.x;
   const void* block_in = nullptr;
   // RB7 residual blocks fused into one kernel each (resblock.cu; PSIM_RB7_FUSED=0: layer-wise A/B)
   static const bool rb7_fused = [] { const char* e = getenv("PSIM_RB7_FUSED"); return !(e && atoi(e) == 0); }();
-  for (size_t li = 0; li < m.layers.size(); ++li) {
+  for (size_t li = first; li < m.layers.size(); ++li) {
     const GemmLayer& g = m.layers[li];
     const bool last = li + 1 == m.layers.size();
     void* out = last ? (void*)ctx->buf.h : ctx->buf.act[li];
@@ -986,6 +987,22 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
     }
     if (predict) {
       g.step = t;
+      // RB7: gather + stem convolution in one kernel (rb7_stem.cu; PSIM_RB7_STEM=0: layer-wise A/B)
+      static const bool rb7_stem = [] { const char* e = getenv("PSIM_RB7_STEM"); return !(e && atoi(e) == 0); }();
+      if (bf16 && rb7_stem && ctx->model.arch == PSIM_ARCH_RB7 && !ctx->model.layers.empty() &&
+          ctx->model.layers[0].K == 128 && ctx->model.layers[0].N == 64) {
+        const GemmLayer& l0 = ctx->model.layers[0];
+        pf.begin(PSIM_KC_LAYER0);
+        launch_rb7_stem(g, (const __nv_bfloat16*)l0.w, l0.bias, (__nv_bfloat16*)ctx->buf.act[0], st);
+        pf.end(PSIM_KC_LAYER0);
+        const int r = run_cnn(ctx, n, 1, ctx->buf.act[0]);
+        if (r) return r;
+        u.step = t;
+        pf.begin(PSIM_KC_UPDATE);
+        launch_update(u, st);
+        pf.end(PSIM_KC_UPDATE);
+        return PSIM_OK;
+      }
       pf.begin(PSIM_KC_GATHER);
       if (bf16) launch_gather_bf16(g, (__nv_bfloat16*)ctx->buf.x, st);
       else launch_gather_f32(g, (float*)ctx->buf.x, st);
