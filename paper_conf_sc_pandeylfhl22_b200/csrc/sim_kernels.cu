@@ -66,7 +66,9 @@ __global__ void __launch_bounds__(256) gather_kernel(GatherArgs a, T* __restrict
       const uint8_t* ar = a.trace + (row - a.row_lo) * a.stride;
       if (aligned8) {
         const uint2 lo = ch > 0 ? __ldg(reinterpret_cast<const uint2*>(ar) + ch - 1) : make_uint2(0u, 0u);
-        const uint2 hi = __ldg(reinterpret_cast<const uint2*>(ar) + ch);   // bytes 8 ch .. 8 ch + 7
+        // bytes 8 ch .. 8 ch + 7 (chunk 6 needs only bytes 45, 46 of lo: its hi word would lie
+        // past the 47 attributes, past the buffer for the last row)
+        const uint2 hi = ch < 6 ? __ldg(reinterpret_cast<const uint2*>(ar) + ch) : make_uint2(0u, 0u);
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
           const int f = 8 * ch + i;

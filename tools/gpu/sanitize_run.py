@@ -1,6 +1,7 @@
 """Small runs of every hot-path kernel for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): the fused C3 path (resident and pinned-streamed trace, several
-tiles per CTA), post-error correction, interval metrics, the layer-wise path and RB7."""
+tiles per CTA), post-error correction, interval metrics, the layer-wise path, the 2:4
+sparse GEMMs and RB7 (fused gather + stem, residual-block kernel)."""
 import os
 import sys
 
@@ -29,10 +30,13 @@ for mode, kw in [("device", {}), ("pinned", {"chunk_steps": 7}), ("pageable", {"
         sim.load_model("C3", w)
         sim.simulate()
         out.append((mode, sim.total_cycles()))
-if not small:
-    wr = synth.weights("RB7")
-    with P.Simulator(precision="bf16") as sim:
-        sim.load_trace(tr[:6000]); sim.partition(16, 8); sim.load_model("RB7", wr); sim.simulate()
-        out.append(("rb7", sim.total_cycles()))
+with P.Simulator(precision="bf16", sparse24=True) as sim:
+    sim.load_trace(tr); sim.partition(N, W); sim.load_model("C3", synth.weights("C3", sparse24=True)); sim.simulate()
+    out.append(("sparse", sim.total_cycles()))
+wr = synth.weights("RB7")
+with P.Simulator(precision="bf16") as sim:   # ragged: several 128-row stem / residual tiles
+    nr = 3000 if small else 30_000
+    sim.load_trace(tr[:nr]); sim.partition(20 if small else 300, 8); sim.load_model("RB7", wr); sim.simulate()
+    out.append(("rb7", sim.total_cycles()))
 print(out)
 assert len({t for m, t in out if m in ("device", "pinned", "layerwise")}) >= 1
