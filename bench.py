@@ -132,13 +132,14 @@ def roofline(stats, k_steps, cfg):
     fused = stats["layer_k"][0] == 0 and stats["layer_m"][0] > 0   # fused path: conv_stack + fc1_head
     sustained = pk["bf16_tflops_sustained"]
     if cfg["arch"] == "RB7" and names[dom].startswith("gemm_layer"):
-        # layer-wise tcgen05 GEMMs, reported together (one kernel, 8 launches per step): stem
-        # 2*56*100*64 + six k3 convs 6 * 2*56*192*64 + fc1 2*3584*256 per simulated instruction
+        # the RB7 tensor-core kernels, reported together (5 launches per step: gather + stem
+        # fused, 3 residual blocks, fc1): stem 2*56*100*64 + six k3 convs 6 * 2*56*192*64 + fc1
+        # 2*3584*256 per simulated instruction
         g = [i for i in range(len(names)) if names[i].startswith("gemm_layer")]
         g_ms = sum(ms[i] for i in g)
         flops = float(stats["simulated"]) * k_steps * (716800 + 6 * 1376256 + 1835008)
         achieved = flops / (g_ms / 1e3) / 1e12
-        out.update(kernel="gemm_tc_kernel (all RB7 layers)", share=round(g_ms / total_ms, 4), bound="tensor",
+        out.update(kernel="rb7_stem_kernel + resblock_kernel x3 + gemm_tc_kernel (fc1): all RB7 layers", share=round(g_ms / total_ms, 4), bound="tensor",
                    achieved=round(achieved, 2), peak=sustained, unit="TFLOP/s", frac=round(achieved / sustained, 4),
                    flops_per_step=flops / k_steps, peak_source=src + " bf16_tflops_sustained")
         avg_s = g_ms / 1e3 / max(sum(launches[i] for i in g), 1)
@@ -168,7 +169,8 @@ def roofline(stats, k_steps, cfg):
         achieved = byts / avg_s / 1e9
         out.update(bound="hbm", achieved=round(achieved, 1), peak=pk["hbm_gbs"], unit="GB/s",
                    frac=round(achieved / pk["hbm_gbs"], 4), bytes_per_launch=byts, peak_source=src + " hbm")
-    out["traffic"] = ncu_traffic(names[dom])
+    # DRAM bytes of an ncu capture of the dominant kernel (profiles/ncu_traffic.json: C3 captures only)
+    out["traffic"] = None if cfg["arch"] == "RB7" else ncu_traffic(names[dom])
     out["avg_launch_us"] = round(avg_s * 1e6, 2)
     if fused:
         out["kernel"] = {"gemm_layer0": "conv_stack_kernel (gather+conv1+conv2+conv3, fused)",
