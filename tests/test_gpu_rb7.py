@@ -2,9 +2,11 @@
 against the oracle, through the C ABI.
 
 RB7 = stem conv 50->64 (k2 s2) + 3 residual blocks y = relu(x + conv_b(relu(conv_a(x))))
-of k3 s1 pad-1 convs + fc1 3584->256 + fc2.  On the GPU the k3 convs run on the
-tcgen05 GEMM with row-shifted TMA loads over a pad-row layout (no im2col) and
-the residual add + ReLU in the epilogue; bf16 operands only.
+of k3 s1 pad-1 convs + fc1 3584->256 + fc2.  On the GPU the row gather is fused with
+the stem (rb7_stem.cu: the stem's A operand is built in shared memory), each residual
+block is one kernel (resblock.cu: 130-row tiles with the k3 halo, the three taps as
+row-shifted smem descriptors, conv_a's output kept on chip, residual add + ReLU in the
+epilogue), fc1 runs on the tcgen05 GEMM; bf16 operands only.
 
 S2: CNN on fixed gathered inputs, bf16 path <= 2e-2 vs the fp64 oracle and
     <= 1e-3 vs the bf16-operand oracle.
@@ -86,3 +88,14 @@ def test_s3_rb7_config5_shape():
         st = sim.stats()
         assert sim.total_cycles() == int(sim.subtrace_cycles().sum()) > 0
     assert st["counted"] == L and st["trace_mode"] == 1 and st["simulated"] == L + 511 * 1000
+
+
+def test_s3_rb7_many_tiles_per_cta():
+    """Several persistent-loop iterations per CTA of the fused gather + stem and residual
+    kernels (4096 sub-traces: 1792 stem / residual tiles of 128 rows on 2 CTAs per SM):
+    decision agreement and raw outputs on sampled sub-traces at both ends and in the
+    middle of the batch."""
+    L, N = 4096 * 48, 4096
+    tr = synth.trace(L, 5077)
+    w = synth.weights("RB7")
+    check_decisions(rb7_decisions(tr, N, w, (0, 1, 2047, 4094, 4095)))
