@@ -637,6 +637,7 @@ static int run_cnn(psim_ctx* ctx, uint64_t n, size_t first = 0, const void* in0 
       pf.begin(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
       launch_resblock((const __nv_bfloat16*)in, (const __nv_bfloat16*)g.w, g.bias, (const __nv_bfloat16*)gb.w, gb.bias,
                       (__nv_bfloat16*)outb, M, ctx->stream);
+      CK(cudaGetLastError());
       pf.end(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
       in = outb;
       ++li;   // conv_b done inside the block kernel
@@ -656,6 +657,7 @@ static int run_cnn(psim_ctx* ctx, uint64_t n, size_t first = 0, const void* in0 
     } else {
       launch_gemm_simt_f32((const float*)in, (const float*)g.w, g.bias, (float*)out, M, g.N, g.K, g.relu, ctx->stream);
     }
+    CK(cudaGetLastError());
     pf.end(PSIM_KC_LAYER0 + (int)std::min<size_t>(li, 3));
     in = out;
   }
@@ -678,7 +680,11 @@ extern "C" int psim_cnn_forward(psim_ctx* ctx, const float* X, uint64_t B, float
     launch_pad_inputs(dX, B, ctx->buf.x, ctx->model.precision == PSIM_BF16, ctx->stream, ctx->model.item_rows,
                       ctx->model.row_off);
     ctx->prof.reset(false, ctx->stream);
-    run_cnn(ctx, B);
+    const int rc2 = run_cnn(ctx, B);
+    if (rc2) {
+      cudaFree(dX);
+      return rc2;
+    }
     e = cudaMemcpyAsync(Y, ctx->buf.y, B * 3 * sizeof(float), cudaMemcpyDeviceToHost, ctx->stream);
   }
   if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
@@ -994,6 +1000,7 @@ extern "C" int psim_simulate(psim_ctx* ctx) {
         const GemmLayer& l0 = ctx->model.layers[0];
         pf.begin(PSIM_KC_LAYER0);
         launch_rb7_stem(g, (const __nv_bfloat16*)l0.w, l0.bias, (__nv_bfloat16*)ctx->buf.act[0], st);
+        CK(cudaGetLastError());
         pf.end(PSIM_KC_LAYER0);
         const int r = run_cnn(ctx, n, 1, ctx->buf.act[0]);
         if (r) return r;
