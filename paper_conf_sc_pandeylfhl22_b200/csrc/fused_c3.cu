@@ -50,8 +50,9 @@ constexpr int W3_OFF = W2_OFF + 32 * 1024;   // 2 atoms [128][64]: ONE K-half of
                                              // (halves alternate with the conv3 MMAs, from L2)
 constexpr int NX = 2;                        // X slots: gathered items in flight
 constexpr int X_OFF = W3_OFF + 32 * 1024;    // NX slots x 2 atoms [128][64]
-constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 4 warps x [32 rows][128 B] (half rows)
-constexpr int BE_OFF = STG_OFF + 16 * 1024;  // uint4 [3 tiles][256 issuer lanes]: block entries staged by cp.async
+constexpr int STG_OFF = X_OFF + NX * 32 * 1024;   // conv3 epilogue staging: 2 groups x 4 warps x [32 rows][128 B]
+                                                  // (EG-B: channels 0..63 of a4 rows, EG-A: 64..127)
+constexpr int BE_OFF = STG_OFF + 32 * 1024;  // uint4 [3 tiles][256 issuer lanes]: block entries staged by cp.async
 constexpr int ER = 8, ED = 4;                // queue-entry ring: items staged ED ahead in ER slots
 constexpr int ER_OFF = BE_OFF + 12 * 1024;   // uint4 [ER items][256 issuer lanes]: queue entries staged by cp.async
 constexpr int BAR_OFF = ER_OFF + ER * 4096;  // mbarriers
@@ -103,6 +104,55 @@ struct ConvArgs {
   __nv_bfloat16* a4;         // [n][14][128]
   long long* dbg;            // optional stage timestamps of CTA 0 (PSIM_DEBUG_TIMING), else nullptr
 };
+
+// conv3 epilogue, one channel half (64 channels = 128 B of an a4 row) of a tile: C3 columns
+// 64 hf .. 64 hf + 63 -> relu(+b3) -> bf16 (TMEM released on read-out), staged in this warp's
+// 4 KB (XOR-swizzled by 16-B chunk), then written out coalesced: one instruction stores four
+// 128-B half rows.  EG-B takes half 0, EG-A half 1 (split so a lone tile's drain -- the G = 8
+// critical path -- is two half-length epilogues in parallel).
+__device__ __forceinline__ void e3_half(uint8_t* stg_base, uint32_t tmem_c3, const float* sb3, uint64_t* c3empty,
+                                        __nv_bfloat16* a4, uint32_t id, int hf, int q, int lane, bool stores) {
+  uint32_t pk[32];
+  {
+    uint32_t r0[32], r1[32];
+    tmem_ld32_nowait(tmem_c3 + 64 * hf, r0);
+    tmem_ld32_nowait(tmem_c3 + 64 * hf + 32, r1);
+    tmem_wait_ld();
+    fence_before();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(c3empty);                // this half of C3 free for the next tile's conv3
+    bias_relu_pack32(r0, sb3 + 64 * hf, pk);
+    bias_relu_pack32(r1, sb3 + 64 * hf + 32, pk + 16);
+  }
+  auto stg = [&](int r, int c) -> uint4* {   // staged half row r (< 32) of this warp, 16-B chunk c (< 8)
+    return reinterpret_cast<uint4*>(stg_base + q * 4096 + r * 128) + (c ^ (r & 7));
+  };
+#pragma unroll
+  for (int c = 0; c < 8; ++c) *stg(lane, c) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+  __syncwarp();
+  if (!stores) return;
+#pragma unroll 4
+  for (int u = 0; u < 8; ++u) {
+    const int rr = 4 * u + (lane >> 3), cc = lane & 7;
+    const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
+    const uint4 v = *stg(rr, cc);
+    if (rid != 0xFFFFFFFFu) reinterpret_cast<uint4*>(a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128 + hf * 64)[cc] = v;
+  }
+  __syncwarp();                                         // staging reads done before it is rewritten
+}
+// the stores of a half staged by e3_half(..., stores = false)
+__device__ __forceinline__ void e3_half_stores(uint8_t* stg_base, __nv_bfloat16* a4, uint32_t id, int hf, int q,
+                                               int lane) {
+  auto stg = [&](int r, int c) -> uint4* { return reinterpret_cast<uint4*>(stg_base + q * 4096 + r * 128) + (c ^ (r & 7)); };
+#pragma unroll 4
+  for (int u = 0; u < 8; ++u) {
+    const int rr = 4 * u + (lane >> 3), cc = lane & 7;
+    const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
+    const uint4 v = *stg(rr, cc);
+    if (rid != 0xFFFFFFFFu) reinterpret_cast<uint4*>(a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128 + hf * 64)[cc] = v;
+  }
+  __syncwarp();
+}
 
 // debug timestamps (build with PSIM_TIMING=1): dbg[tile * 256 + slot] = clock64()
 // for CTA 0, first 4 tiles of the step named by $PSIM_DEBUG_TIMING
@@ -177,7 +227,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   uint64_t* c2empty = bars + 12;   // [2] commit: the conv3 MMAs reading the slot's A3 done
   uint64_t* a3full = bars + 14;    // [2] 4 (EG-B): A3 (bf16) written into the C2 slot
   uint64_t* c3full = bars + 16;    //     commit
-  uint64_t* c3empty = bars + 17;   //     4 (EG-B)
+  uint64_t* c3empty = bars + 17;   //     8 (EG-B: C3 columns 0..63, EG-A: 64..127)
   uint64_t* wbar = bars + 18;      //     weights + biases landed
   uint64_t* w3full = bars + 21;    //     W3 K-half landed (TMA)
   uint64_t* w3empty = bars + 22;   //     commit: the conv3 MMAs of that half are done
@@ -191,7 +241,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
       mbar_init(c1full + i, 1); mbar_init(c1empty + i, 1); mbar_init(a2full + i, 4);
       mbar_init(c2full + i, 1); mbar_init(c2empty + i, 1); mbar_init(a3full + i, 4);
     }
-    mbar_init(c3full, 1); mbar_init(c3empty, 4);
+    mbar_init(c3full, 1); mbar_init(c3empty, 8);
     mbar_init(wbar, 1);
     mbar_init(w3full, 1); mbar_init(w3empty, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -357,7 +407,25 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
           conv2_epilogue(tmem, lane_base, sb2, c2full, a3full, it, j >> 1, lane);
           if (q == 0) PSIM_TS(j == 1 ? 59 : 63);
         }
+        if (j == 1 && it > 0) {   // channels 64..127 of the previous tile's conv3 (complete by now: its last
+                                  // MMAs were issued before this tile's conv2 position 0): read out + staged
+          wait_full(c3full, it - 1);
+          fence_after();
+          e3_half(sm + cs::STG_OFF + 16384, tmem + lane_base + cs::TMEM_C3, sb3, c3empty, a.a4, 0u, 1, q, lane, false);
+        }
       }
+      if (it > 0) {             // ... and written out once this tile's conv1 epilogues are done
+        const uint32_t bi = (tl - gridDim.x) * cs::TILE + q * 32 + lane;
+        e3_half_stores(sm + cs::STG_OFF + 16384, a.a4, bi < nblocks ? a.blocks[bi].x : 0xFFFFFFFFu, 1, q, lane);
+      }
+    }
+    if (it > 0) {               // the last tile's half: both halves drain in parallel (EG-B takes 0..63)
+      const uint32_t tl_last = blockIdx.x + (it - 1) * gridDim.x;
+      const uint32_t bi = tl_last * cs::TILE + q * 32 + lane;
+      const uint32_t id = bi < nblocks ? a.blocks[bi].x : 0xFFFFFFFFu;
+      wait_full(c3full, it - 1);
+      fence_after();
+      e3_half(sm + cs::STG_OFF + 16384, tmem + lane_base + cs::TMEM_C3, sb3, c3empty, a.a4, id, 1, q, lane, true);
     }
   } else if (warp < 8) {   // ============================ EG-B: conv2 position 1 + conv3 epilogues
     setmaxnreg_inc<cs::REG_EPI>();
@@ -366,55 +434,16 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     const int q = warp & 3;
     const int m = q * 32 + lane;
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
-    // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p]: both halves are read out of TMEM first
-    // (C3 released at once for the next tile's conv3), then one half row (64 channels,
-    // 128 B) at a time is staged in this warp's 4 KB of the staging buffer (XOR-swizzled
-    // by 16-B chunk) and written out coalesced: one instruction stores four 128-B half rows.
-    auto e3 = [&](uint32_t it, uint32_t tl) {
+    // C3 (128 fp32) -> relu(+b3) -> bf16 -> a4[b][p], channels 0..63 here (e3_half); EG-A
+    // drains channels 64..127 after its conv2 position-0 epilogue of the next tile.
+    auto e3 = [&](uint32_t it, uint32_t tl) {   // channels 0..63 (EG-A takes 64..127)
       const uint32_t bi = tl * cs::TILE + m;
       const uint32_t id = bi < nblocks ? a.blocks[bi].x : 0xFFFFFFFFu;
       if (q == 0) PSIM_TS(64);
       wait_full(c3full, it);                          // conv3 accumulated
       if (q == 0) PSIM_TS(65);
       fence_after();
-      uint32_t pk[64];
-      {
-        uint32_t r0[32], r1[32];
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 32, r1);
-        tmem_wait_ld();
-        bias_relu_pack32(r0, sb3, pk);
-        bias_relu_pack32(r1, sb3 + 32, pk + 16);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 64, r0);
-        tmem_ld32_nowait(tmem + lane_base + cs::TMEM_C3 + 96, r1);
-        tmem_wait_ld();
-        fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(c3empty);          // C3 TMEM free for the next tile's conv3
-        bias_relu_pack32(r0, sb3 + 64, pk + 32);
-        bias_relu_pack32(r1, sb3 + 96, pk + 48);
-      }
-      if (q == 0) PSIM_TS(68);
-      auto stg = [&](int r, int c) -> uint4* {   // staged half row r (< 32) of this warp, 16-B chunk c (< 8)
-        return reinterpret_cast<uint4*>(sm + cs::STG_OFF + q * 4096 + r * 128) + (c ^ (r & 7));
-      };
-#pragma unroll
-      for (int half = 0; half < 2; ++half) {
-#pragma unroll
-        for (int c = 0; c < 8; ++c)
-          *stg(lane, c) = make_uint4(pk[32 * half + 4 * c], pk[32 * half + 4 * c + 1], pk[32 * half + 4 * c + 2],
-                                     pk[32 * half + 4 * c + 3]);
-        __syncwarp();
-#pragma unroll 4
-        for (int u = 0; u < 8; ++u) {
-          const int rr = 4 * u + (lane >> 3), cc = lane & 7;
-          const uint32_t rid = __shfl_sync(0xffffffffu, id, rr);
-          const uint4 v = *stg(rr, cc);
-          if (rid != 0xFFFFFFFFu)
-            reinterpret_cast<uint4*>(a.a4 + ((uint64_t)(rid >> 4) * 14 + (rid & 15)) * 128 + half * 64)[cc] = v;
-        }
-        __syncwarp();                                 // staging reads done before it is rewritten
-      }
+      e3_half(sm + cs::STG_OFF, tmem + lane_base + cs::TMEM_C3, sb3, c3empty, a.a4, id, 0, q, lane, true);
       if (q == 0) PSIM_TS(66);
     };
     uint32_t it = 0, prev_tl = 0;
