@@ -36,3 +36,22 @@ def test_roofline_frac_reproducible():
     assert r["kernel"].startswith("conv_stack")
     step_s = 111.0 / 1e3 / steps
     assert abs(r["step"]["frac"] - (bps * 247_808 + n * 1536) / step_s / 1e12 / peak) < 1e-3
+
+
+def test_roofline_rb7_counts_all_tensor_kernels():
+    """RB7 (config 5): the fused gather + stem, residual-block and fc1 kernels are reported
+    together against 10.81 MFLOP per simulated instruction, with no DRAM
+    figure borrowed from a C3 capture."""
+    steps, n = 100, 4096
+    st = {"kernel_names": ["gemm_layer0", "gemm_layer1", "gemm_layer2", "gemm_layer3", "gather", "update",
+                           "head", "other"],
+          "kernel_ms": [10.0, 20.0, 0, 30.0, 0, 5.0, 1.0, 0.5],
+          "kernel_launches": [steps, steps, 0, 3 * steps, 0, steps, steps, 2],
+          "k_hist": [0] * 112, "layer_m": [n * 58, n * 58, 0, n], "layer_n": [64, 64, 0, 256],
+          "layer_k": [128, 192, 0, 3712], "subtraces": n, "simulated": n * steps, "steps": steps, "sim_ms": 66.5}
+    r = bench.roofline(st, 1, {"arch": "RB7", "precision": "bf16"})
+    flop = n * steps * (2 * 56 * 100 * 64 + 6 * 2 * 56 * 192 * 64 + 2 * 3584 * 256)
+    assert flop == n * steps * 10_809_344
+    want = flop / 60e-3 / 1e12 / r["peak"]
+    assert abs(r["frac"] - want) < 1e-3
+    assert "resblock" in r["kernel"] and r["traffic"] is None
