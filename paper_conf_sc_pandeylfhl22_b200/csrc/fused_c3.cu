@@ -161,9 +161,23 @@ __device__ __forceinline__ void e3_half_stores(uint8_t* stg_base, __nv_bfloat16*
   do {                                                                                                 \
     if (a.dbg && blockIdx.x == 0 && it < 4 && lane == 0) a.dbg[it * 256 + (slot)] = clock64();        \
   } while (0)
+// per-CTA span of a kernel: dbg[1024 + (kernel * 160 + cta) * 4 + {0 entry, 1 after the PDL
+// wait, 2 end, 3 tiles}] = %globaltimer (ns, comparable across SMs)
+#define PSIM_CTA_TS(kern, slot, val)                                                                   \
+  do {                                                                                                 \
+    if (a.dbg && threadIdx.x == 0 && blockIdx.x < 160) a.dbg[1024 + ((kern) * 160 + blockIdx.x) * 4 + (slot)] = (val); \
+  } while (0)
+__device__ __forceinline__ long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return (long long)t;
+}
 #else
 #define PSIM_TS(slot) \
   do {                \
+  } while (0)
+#define PSIM_CTA_TS(kern, slot, val) \
+  do {                               \
   } while (0)
 #endif
 
@@ -218,6 +232,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
+  PSIM_CTA_TS(0, 0, gtimer());
   uint64_t* xfull = bars + 24;     // [NX] 4 gather warps (arrive.expect_tx) + the gathered rows (complete_tx)
   uint64_t* xempty = bars + 28;    // [NX] commit
   uint64_t* c1full = bars + 4;     // [2] commit: conv1 of the slot's item done
@@ -268,6 +283,8 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   grid_dep_launch_dependents();
   const uint32_t nblocks = *a.nblocks;
   const uint32_t ntiles = (nblocks + cs::TILE - 1) / cs::TILE;
+  PSIM_CTA_TS(0, 1, gtimer());
+  PSIM_CTA_TS(0, 3, (long long)((ntiles + gridDim.x - 1 - blockIdx.x) / gridDim.x));
   if (blockIdx.x == 0 && tid == 0) *a.next_count = 0;
   if (warp <= cs::MMA_WARP) mbar_wait(wbar, 0);   // weights (MMA issuer) and biases (epilogues) resident
   // register budget (setmaxnreg redistributes the launch allocation of 640 x 96; with
@@ -585,6 +602,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
   }
   fence_before();
   __syncthreads();
+  PSIM_CTA_TS(0, 2, gtimer());
   if (warp == cs::MMA_WARP) {
     fence_after();
     tmem_dealloc(tmem, cs::TMEM_COLS);
@@ -640,6 +658,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   float* sT = reinterpret_cast<float*>(sm + fh::T_OFF);
+  PSIM_CTA_TS(1, 0, gtimer());
   float* sW2 = reinterpret_cast<float*>(sm + fh::W2_OFF);
   int* sP = reinterpret_cast<int*>(sm + fh::P_OFF);
   unsigned int* sHist = reinterpret_cast<unsigned int*>(sm + fh::H_OFF);
@@ -714,6 +733,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     }
   }
   grid_dep_wait();
+  PSIM_CTA_TS(1, 1, gtimer());
   if (warp >= 2 && warp < 6) mbar_wait(cbar, 0);   // epilogue warps read T and fc2 from smem
 
   if (warp == 0) {
@@ -926,6 +946,14 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     if (sHist[k]) atomicAdd(a.u.st.k_hist + k, (unsigned long long)sHist[k]);
   fence_before();
   __syncthreads();
+  PSIM_CTA_TS(1, 2, gtimer());
+#ifdef PSIM_TIMING
+  {
+    int nt = 0, pmax = 0;
+    for (uint32_t tt = t0; tt < tend; tt += tstep) { ++nt; pmax = max(pmax, tileP_of(tt)); }
+    PSIM_CTA_TS(1, 3, (long long)(nt * 256 + pmax));
+  }
+#endif
   if constexpr (kPair) cluster_sync();   // the peer no longer signals this CTA's barriers
   if (warp == 1) {
     fence_after();
@@ -1146,25 +1174,34 @@ void launch_fused_init(FusedC3& f, const int64_t* ws, uint64_t n, cudaStream_t s
 // pipeline event of its first 4 tiles of that step (dumped to
 // $PSIM_DEBUG_TIMING_OUT by fused_dump_debug).  Off by default.
 static long long* g_dbg = nullptr;
+constexpr int kDbgWords = 1024 + 2 * 160 * 4;   // CTA-0 slots, then per-CTA spans
 static int64_t g_dbg_step = -2;
 static long long* debug_buffer(int64_t step) {
   if (g_dbg_step == -2) {
     const char* e = getenv("PSIM_DEBUG_TIMING");
     g_dbg_step = e ? atoll(e) : -1;
-    if (g_dbg_step >= 0) { cudaMalloc(&g_dbg, 4 * 256 * 8); cudaMemset(g_dbg, 0, 4 * 256 * 8); }
+    if (g_dbg_step >= 0) { cudaMalloc(&g_dbg, 2 * kDbgWords * 8); cudaMemset(g_dbg, 0, 2 * kDbgWords * 8); }
   }
-  return (g_dbg_step >= 0 && step == g_dbg_step) ? g_dbg : nullptr;
+  if (g_dbg_step < 0) return nullptr;
+  if (step == g_dbg_step) return g_dbg;
+  return step == g_dbg_step + 1 ? g_dbg + kDbgWords : nullptr;   // the next step: per-CTA spans
 }
 void fused_dump_debug() {
   const char* out = getenv("PSIM_DEBUG_TIMING_OUT");
   if (!g_dbg || !out) return;
-  long long h[4 * 256];
+  static long long h[2 * kDbgWords];
   cudaMemcpy(h, g_dbg, sizeof h, cudaMemcpyDeviceToHost);
   FILE* f = fopen(out, "w");
   if (!f) return;
   for (int t = 0; t < 4; ++t)
     for (int sidx = 0; sidx < 256; ++sidx)
       if (h[t * 256 + sidx]) fprintf(f, "%d %d %lld\n", t, sidx, h[t * 256 + sidx]);
+  for (int st = 0; st < 2; ++st)   // per-CTA spans: "cta <kernel> <cta> <entry> <after wait> <end> <tiles>"
+    for (int k = 0; k < 2; ++k)     // kernel 0/1 = conv_stack / fc1_head of the step, 2/3 of the next step
+      for (int c = 0; c < 160; ++c) {
+        const long long* r = h + st * kDbgWords + 1024 + (k * 160 + c) * 4;
+        if (r[0]) fprintf(f, "cta %d %d %lld %lld %lld %lld\n", k + 2 * st, c, r[0], r[1], r[2], r[3]);
+      }
   fclose(f);
 }
 
