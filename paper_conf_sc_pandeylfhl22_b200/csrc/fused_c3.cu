@@ -87,7 +87,7 @@ struct ConvArgs {
   const uint32_t* nblocks;   // count of this step's list
   uint32_t* next_count;      // the other step parity's counter, reset here
   const __nv_bfloat16* trace16;   // [rows + 1][48] bf16 operand rows (attributes at cols 0..46), row `rows` zero
-  uint32_t zero_row;         // index of the all-zero trace16 row (padding rows of the input)
+  uint32_t zero_row;         // gather row index of the padding rows of the input (kPadRow: out of bounds, TMA zero fill)
   int64_t row_lo;
   const int64_t* ws;
   const int64_t* clock;
@@ -480,7 +480,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // position j = n % 4 of this CTA's tile n / 4: input rows R = 8p + 2j + h (h = 0, 1;
     // PAPER.md:93 row order) of the tile's 128 blocks (b, p).
     // Lane l of issuer warp wq BUILDS the row of block m = 16 wq + (l & 15), h = l >> 4:
-    // padding (R > k) -> the all-zero trace16 row past the rank's rows; R = 0 -> the
+    // padding (R > k) -> row kPadRow past the tensor (zero-filled by the TMA); R = 0 -> the
     // current instruction; context rows newest first -> the row of queue entry k - R (R6),
     // with the time features age / remaining-to-complete / remaining-to-retire (R2) in
     // chunk 6 (cols 48..55) of its SW128 operand row.  The metadata chain block entry
@@ -1298,7 +1298,11 @@ bool fused_make_weight_maps(FusedC3& f) {
 }
 
 bool fused_make_trace_map(FusedC3& f, uint64_t rows) {
-  f.zero_row = (uint32_t)rows;
+  // padding rows of the gathered input (rows R > k) use a row index past the
+  // tensor: the TMA zero-fills out-of-bounds rows without reading memory.  (Pointing them at
+  // one all-zero trace16 row made that 96-B line an L2 hot spot -- ~230k reads per step at
+  // config 3, all served by one L2 slice: conv_stack 131 -> 114 ms per run without it.)
+  f.zero_row = kPadRow;
   // 96-B rows (48 bf16: 47 attributes + 0); a 48-column box lands in chunks 0..5 of the
   // 128-B SWIZZLE_128B operand rows, chunks 6 (time features) and 7 (zero) are the gather's
   EncodeTiledFn fn = encode_fn2();

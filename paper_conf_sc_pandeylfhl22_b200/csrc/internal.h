@@ -21,6 +21,7 @@ constexpr int kFeatPad = 64;    // device row width: features padded with zeros 
 constexpr int kQStride = 112;   // queue entries reserved per sub-trace (cap <= 110, +1 push)
 constexpr int kLatMax = 4095;   // R7
 constexpr int kTimeMax = 65535; // R7
+constexpr uint32_t kPadRow = 0x7FFF0000u;   // gather4 row past any trace16 tensor: TMA zero fill
 
 // One GEMM layer of the lowered CNN: out[M][N] = act(A[M][K] . W[N][K]^T + b[N]).
 // Convolutions with k = s = 2 read A as the row-pair reshape of the previous
@@ -229,7 +230,8 @@ struct FusedC3 {
                                       // cohorts with disjoint SM shares run side by side
   CUtensorMap mapW1, mapW2, mapW3;    // TMA maps of the resident conv weights (SWIZZLE_128B)
   CUtensorMap mapX;                   // TMA gather4 map of trace16 [rows + 1][48] (box 48 x 1, SWIZZLE_128B)
-  uint32_t zero_row = 0;              // trace16 row that is all zero (= the rank's row count)
+  uint32_t zero_row = 0;              // gather row index of the input's padding rows (kPadRow: out of
+                                      // bounds of mapX, zero-filled by the TMA)
 };
 void launch_fused_init(FusedC3& f, const int64_t* ws, uint64_t n, cudaStream_t st);
 // block list / P_tile of step 0 of a pass whose sub-traces start from a non-empty
@@ -249,7 +251,7 @@ void launch_fc1_head(FusedC3& f, const UpdateArgs& u, const int64_t* e, int64_t 
 bool fused_make_maps(FusedC3& f, uint64_t n);
 int sm_count();   // SMs of the current device
 bool fused_make_weight_maps(FusedC3& f);
-// gather4 map of f.trace16 with rows + 1 rows (the last one zero); sets f.zero_row
+// gather4 map of f.trace16 with rows + 1 rows (the last one zero); sets f.zero_row = kPadRow
 bool fused_make_trace_map(FusedC3& f, uint64_t rows);
 void fused_dump_debug();
 
