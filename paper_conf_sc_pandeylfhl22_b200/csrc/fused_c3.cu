@@ -617,17 +617,22 @@ constexpr int STAGES = 4;
 constexpr int T_STRIDE = 260;                 // padded rows of the constant table (bank spread, 16-B rows)
 constexpr int T_OFF = STAGES * STAGE;         // float [15][257]
 constexpr int W2_OFF = T_OFF + 15 * T_STRIDE * 4;   // float [3][256] + bias[3]
-constexpr int Y_OFF = W2_OFF + (3 * 256 + 4) * 4;   // float [128][3]
-constexpr int P_OFF = Y_OFF + 2 * 128 * 3 * 4;      // int [2][16] tile scan scratch per update group
-constexpr int H_OFF = P_OFF + 32 * 4;               // uint [112] k histogram of this CTA
+#ifndef PSIM_FC1_UPD_GROUPS
+#define PSIM_FC1_UPD_GROUPS 2
+#endif
+constexpr int UPD_GROUPS = PSIM_FC1_UPD_GROUPS;   // update groups of 4 warps, tiles round-robin
+constexpr int Y_OFF = W2_OFF + (3 * 256 + 4) * 4;   // float [UPD_GROUPS][128][3]: y of tile t in buffer t % UPD_GROUPS
+constexpr int P_OFF = Y_OFF + UPD_GROUPS * 128 * 3 * 4;      // int [UPD_GROUPS][16] tile scan scratch per update group
+constexpr int H_OFF = P_OFF + UPD_GROUPS * 16 * 4;  // uint [112] k histogram of this CTA
 constexpr int BAR_OFF = (H_OFF + 112 * 4 + 7) & ~7;
+static_assert(8 * (4 + 4 + 2 + 2 + 1 + 2 * UPD_GROUPS) + 4 <= 256, "barrier area");
 constexpr int SMEM = BAR_OFF + 256 + 1024;
 // pair mode (fc1 on 2-SM MMAs): a cluster of two CTAs computes two tiles with one
 // tcgen05.mma.cta_group::2 (M = 256): each CTA stages its own tile's a4 rows and HALF of the
 // W_fc1 slice (N rows 128 r .. 128 r + 127), so the W_fc1 stream per SM halves; smaller
 // stages (32 KB) -> 6 of them in the same 192 KB
 constexpr int PSTAGE = A_BYTES + B_BYTES / 2, PSTAGES = (STAGES * STAGE) / PSTAGE;
-constexpr int THREADS = 448;   // warp 0 TMA, 1 MMA, 2-5 epilogue (F -> y), 6-9 / 10-13 update groups (even / odd tiles)
+constexpr int THREADS = 192 + 128 * UPD_GROUPS;   // warp 0 TMA, 1 MMA, 2-5 epilogue (F -> y), 6.. update groups (4 warps each)
 }  // namespace fh
 
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
@@ -684,10 +689,12 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   };
 
   uint64_t* cbar = tempty + 2;   // constant table + fc2 landed (bulk copies)
-  uint64_t* yfull = cbar + 1;    // [2] epilogue -> update: y of a tile in sY[buf]
-  uint64_t* yempty = yfull + 2;  // [2] update -> epilogue: sY[buf] consumed
+  // y of tile it in sY[it % UPD_GROUPS], consumed by update group it % UPD_GROUPS (so one
+  // buffer's phases are always consumed in order by one group)
+  uint64_t* yfull = cbar + 1;                   // [UPD_GROUPS] epilogue -> update
+  uint64_t* yempty = yfull + fh::UPD_GROUPS;    // [UPD_GROUPS] update -> epilogue: consumed
   float* sY = reinterpret_cast<float*>(sm + fh::Y_OFF);
-  tmem_slot = reinterpret_cast<uint32_t*>(yempty + 2);
+  tmem_slot = reinterpret_cast<uint32_t*>(yempty + fh::UPD_GROUPS);
   if (tid < 3) sW2[768 + tid] = a.b2[tid];
   for (int idx = tid; idx < 112; idx += fh::THREADS) sHist[idx] = 0;
   if (tid == 0) {
@@ -695,7 +702,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     // pair mode: tempty of the even CTA collects the epilogue warps of both CTAs
     for (int i = 0; i < 2; ++i) { mbar_init(tfull + i, 1); mbar_init(tempty + i, kPair ? 8 : 4); }
     mbar_init(cbar, 1);
-    for (int i = 0; i < 2; ++i) { mbar_init(yfull + i, 4); mbar_init(yempty + i, 4); }
+    for (int i = 0; i < fh::UPD_GROUPS; ++i) { mbar_init(yfull + i, 4); mbar_init(yempty + i, 4); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     mbar_expect_tx(cbar, 15 * 1024 + 3 * 1024);
     for (int r = 0; r < 15; ++r) bulk_g2s(sT + r * fh::T_STRIDE, a.T + r * 256, 1024, cbar);
@@ -805,7 +812,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t it = 0;
     for (uint32_t tt = t0; tt < tend; tt += tstep, ++it) {
-      const int acc = it & 1, yb = it & 1;
+      const int acc = it & 1, yb = it % fh::UPD_GROUPS;
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const int ptile = tileP_of(tt);
       const int kb = b < n ? a.u.st.count[b] : 0;   // read before this tile's update (y handoff orders it)
@@ -859,7 +866,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
           else mbar_arrive(tempty + acc);
         }
       }
-      wait_empty(yempty + yb, it >> 1);
+      wait_empty(yempty + yb, it / fh::UPD_GROUPS);
       float* yrow = sY + (yb * 128 + m) * 3;
       yrow[0] = y0; yrow[1] = y1; yrow[2] = y2;
       __syncwarp();
@@ -872,8 +879,8 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
     const int m = q * 32 + lane;
     int* sPg = sP + grp * 16;
     uint32_t it = grp;
-    for (uint32_t tt = t0 + grp * tstep; tt < tend; tt += 2 * tstep, it += 2) {
-      const int yb = it & 1;
+    for (uint32_t tt = t0 + grp * tstep; tt < tend; tt += fh::UPD_GROUPS * tstep, it += fh::UPD_GROUPS) {
+      const int yb = it % fh::UPD_GROUPS;   // == grp
       const uint64_t b = (uint64_t)tt * fh::BM + m;
       const bool inb = b < n;
       if (q == 0) PSIM_TS(145);
@@ -889,7 +896,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       QBatch first;
       if (active) load_qbatch(a.u.st, b, kb, first);   // (an L2 prefetch of the rest of the queue here: no gain)
       const int pb = min((kb + 8) >> 3, 14);
-      wait_full(yfull + yb, it >> 1);
+      wait_full(yfull + yb, it / fh::UPD_GROUPS);
       if (q == 0) PSIM_TS(146);
       const float* yrow = sY + (yb * 128 + m) * 3;
       const float y0 = yrow[0], y1 = yrow[1], y2 = yrow[2];
