@@ -95,6 +95,7 @@ struct ConvArgs {
   const uint4* q;
   int64_t step;
   uint64_t qn;               // sub-traces (entry stride of the entry-major queue)
+  int rows_keep;             // gathered rows evict_last (small slices: the live context window fits L2)
   const __nv_bfloat16* w1;   // [64][128]
   const __nv_bfloat16* w2;   // [128][128]
   const __nv_bfloat16* w3;   // [128][256]
@@ -503,7 +504,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     // trace rows are streamed through L2 with evict_first: the step's context rows
     // (~145 MB at config 3, G = 1) exceed L2 and would otherwise push out the queue
     // entries, states and a4 rows that are reused within the step
-    const uint64_t pol = l2_policy_evict_first();
+    const uint64_t pol = a.rows_keep ? l2_policy_evict_last() : l2_policy_evict_first();
     const uint4 kNoBlock = make_uint4(0xFFFFFFFFu, 0u, 0u, 0u);
     auto row_R = [&](const uint4& be, uint32_t n) -> int { return (int)(be.x & 15) * 8 + 2 * (int)(n & 3) + hh; };
     // Metadata pipeline, all through lane-private smem rings filled by cp.async (no register
@@ -1228,6 +1229,18 @@ void launch_conv_stack(FusedC3& f, const GatherArgs& g, int64_t step, uint64_t n
   a.q = g.q;
   a.step = step;
   a.qn = g.qn ? g.qn : g.n;
+  // L2 policy of the gathered trace rows: a sub-trace's context rows are re-read every step while
+  // they stay in its queue (~25 steps).  Up to 16384 sub-traces per launch the live window
+  // (~25 rows x 96 B each, <= 40 MB) fits L2 beside the queue and a4: evict_last (+1 % at the
+  // G = 4 / 8 slices); at config 3 on one GPU (157 MB per step) the rows would push out the
+  // queue entries and a4 rows reused within the step: evict_first (evict_last: -4 %, any
+  // evict_last fraction 0.25..0.75: -3..-4 %, evict_normal: -24 %; tools/gpu/abe.sh, frac.sh).
+  // PSIM_ROW_POLICY=first|last overrides (experiments).
+  static const int row_policy = [] {
+    const char* e = getenv("PSIM_ROW_POLICY");
+    return !e ? -1 : (e[0] == 'l' ? 1 : 0);
+  }();
+  a.rows_keep = row_policy >= 0 ? row_policy : (n <= 16384 ? 1 : 0);
   a.w1 = f.w1; a.w2 = f.w2; a.w3 = f.w3;
   a.b1 = f.b1; a.b2 = f.b2; a.b3 = f.b3;
   a.a4 = f.a4;
