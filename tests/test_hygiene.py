@@ -4,6 +4,8 @@
   of the CUDA batched-copy calls that are closed on the GPU pool (they raised a
   GPU fault there).  The names are assembled from pieces so this file does not
   contain them either.
+* No script that travels to the GPU box invokes the CUDA memory-checker tool, which
+  is closed on the GPU pool too (runs under it left GPUs needing a reset).
 * No ELF binary is tracked in git (experiment builds stay out of history).
 """
 import os
@@ -48,6 +50,23 @@ def test_no_closed_copy_calls_anywhere():
                 if n in data:
                     hits.append(f"{os.path.relpath(path, ROOT)}: {n.decode()}")
     assert not hits, "closed CUDA calls named in: " + "; ".join(hits)
+
+
+_TOOL = "compute" + "-" + "sanitizer"
+
+
+def test_no_memory_checker_invocations():
+    hits = []
+    for dp, dns, fns in os.walk(ROOT):
+        dns[:] = [d for d in dns if d not in _SKIP_DIRS]
+        for fn in fns:
+            if not fn.endswith((".sh", ".py", ".c", ".cu", ".cuh", ".h")):
+                continue
+            path = os.path.join(dp, fn)
+            with open(path, "rb") as f:
+                if _TOOL.encode() in f.read():
+                    hits.append(os.path.relpath(path, ROOT))
+    assert not hits, "memory-checker tool invoked in: " + "; ".join(hits)
 
 
 def test_no_tracked_elf_binaries():

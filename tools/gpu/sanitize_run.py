@@ -1,5 +1,5 @@
-"""Small runs of every hot-path kernel for compute-sanitizer (memcheck / racecheck /
-synccheck / initcheck): the fused C3 path (resident and pinned-streamed trace, several
+"""Small runs of every hot-path kernel (the workload of round 2's memory-checker runs, see
+profiles/r02_sanitizer.md; that tool is now closed on the GPU pool): the fused C3 path (resident and pinned-streamed trace, several
 tiles per CTA), post-error correction, interval metrics, the layer-wise path, the 2:4
 sparse GEMMs and RB7 (fused gather + stem, residual-block kernel)."""
 import os
