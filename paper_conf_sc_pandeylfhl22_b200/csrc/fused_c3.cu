@@ -906,8 +906,17 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
       int pnext = 0, knext = 0;
       if (active) {
         bool stopped = false;
+        long long* uts = nullptr;
+#ifdef PSIM_TIMING
+        if (a.dbg && blockIdx.x == 0 && it < 4 && q == 0 && lane == 0) uts = a.dbg + it * 256 + 160;   // slots 160..172
+        {
+          const unsigned am = __activemask();
+          const int kmx = __reduce_max_sync(am, kb);
+          if (uts) uts[15] = kmx;   // slot 175
+        }
+#endif
         const int knew = update_subtrace_thread(a.u, b, ws, s_b, nsteps, kb, clock, rmin, first, run_head, y0, y1, y2, sHist,
-                                                &stopped);
+                                                &stopped, uts);
         if (a.u.step + 1 < nsteps && !stopped) {
           pnext = (knew + 8) >> 3;                 // ceil((k+1)/8)
           knext = knew;

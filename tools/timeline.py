@@ -31,6 +31,9 @@ names.update({128: "tma start", 129: "tma end", 132: "mma wait tempty", 133: "mm
               150: "u2 bnd", 151: "u3 end", 152: "u4 ret", 154: "kmax(warp)", 155: "lanes rmin-clock<=8",
               156: "b0 done", 157: "b1 issued", 158: "b1 done", 159: "b2 issued", 160: "b2 done", 161: "b3 issued",
               162: "b3 done", 163: "b4 issued", 164: "b4 done"})
+names.update({160: "U entry", 161: "U fastdone", 162: "U b0 start", 163: "U b0 done", 164: "U b1 start", 165: "U b1 done",
+              166: "U b2 start", 167: "U b2 done", 168: "U b3 start", 169: "U b3 done", 170: "U b4 start", 171: "U b4 done",
+              172: "U scanned", 175: "kmax"})
 
 d = collections.defaultdict(dict)
 spans = collections.defaultdict(dict)   # kernel -> cta -> (entry, after wait, end, tiles) [globaltimer ns]
@@ -42,7 +45,7 @@ for line in open(sys.argv[1]):
     t, slot, v = map(int, line.split())
     d[t][slot] = v
 for lo, hi, title in ((0, 128, "conv_stack"), (128, 256, "fc1_head")):
-    VALS = (154, 155)   # plain values, not timestamps
+    VALS = (154, 155, 175)   # plain values, not timestamps
     vals = [v for t in d for sl, v in d[t].items() if lo <= sl < hi and sl not in VALS]
     if not vals:
         continue
