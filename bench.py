@@ -370,6 +370,11 @@ def main():
 
     torch.cuda.set_device(local_rank)
     if world > 1:
+        # NCCL's communicator-init lines (rank / nranks / transport) on stderr, so a multi-GPU
+        # run shows its ranks; stdout keeps the one JSON line
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     nccl_id = None
     if world > 1:
@@ -448,6 +453,8 @@ def main():
             "vs_baseline": None, "dtype": cfg["precision"], "data": "synthetic", "config": config,
             "total_cycles": total, "e2e": e2e, "gpu_launches": int(sum(stats["kernel_launches"])),
             "clocks": clocks}
+    if world > 1:   # the final ncclAllReduce of the cycle total: ranks of the library's communicator
+        line["comm"] = {"backend": "nccl", "ranks": int(stats.get("comm_ranks", 0)), "world_size": world}
     if rank == 0:
         line["roofline"] = roofline(stats, args.steps, cfg) if sum(stats["kernel_ms"]) > 0 else None
         line["stats"] = {k: stats[k] for k in ("steps", "simulated", "counted", "stalls", "subtraces", "corrected",
