@@ -231,7 +231,7 @@ __global__ void __launch_bounds__(cs::THREADS, 1)
     conv_stack_kernel(ConvArgs a, const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2,
                       const __grid_constant__ CUtensorMap tmW3, const __grid_constant__ CUtensorMap tmX) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sm = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1024-B aligned; stays in the shared window (LDS/STS, not generic LD/ST)
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + cs::BAR_OFF);
   PSIM_CTA_TS(0, 0, gtimer());
   uint64_t* xfull = bars + 24;     // [NX] 4 gather warps (arrive.expect_tx) + the gathered rows (complete_tx)
@@ -662,7 +662,7 @@ __global__ void __launch_bounds__(fh::THREADS, 1)
   constexpr int kStages = kPair ? fh::PSTAGES : fh::STAGES;
   constexpr int kStage = kPair ? fh::PSTAGE : fh::STAGE;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sm = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1024-B aligned; stays in the shared window (LDS/STS, not generic LD/ST)
   float* sT = reinterpret_cast<float*>(sm + fh::T_OFF);
   PSIM_CTA_TS(1, 0, gtimer());
   float* sW2 = reinterpret_cast<float*>(sm + fh::W2_OFF);

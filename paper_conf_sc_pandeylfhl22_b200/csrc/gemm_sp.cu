@@ -66,7 +66,7 @@ __global__ void __launch_bounds__(192, 1)
                    void* __restrict__ C, int64_t M, int K, int n_out, int relu, int c_f32) {
   using Cfg = SpCfg<MH>;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);   // 1024-B aligned; stays in the shared window (LDS/STS, not generic LD/ST)
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + Cfg::STAGES * Cfg::STAGE);
   uint64_t* empty = full + Cfg::STAGES;
   uint64_t* tfull = empty + Cfg::STAGES;
